@@ -1,0 +1,211 @@
+/*
+ * ugache.h -- C ABI of the B200-native UGache factored-embedding-extraction library.
+ *
+ * Citations "P:n" are lines of the paper text (PAPER.md of dblp/paper_conf_sosp_songz0c23,
+ * "UGache: A Unified GPU Cache for Embedding-based Deep Learning", SOSP'23).
+ *
+ * The hot path (ugache_extract) is the paper's extract() (section 3.2) executed
+ * with the factored extraction mechanism (section 5.3): every key is located
+ * through this GPU's location table (the per-GPU "hashtable" of <GPU_i, Offset>),
+ * keys are grouped by source, SMs dedicated to each non-local source (host
+ * DRAM over PCIe, each peer GPU over NVLink/NVSwitch) copy their group, and local HBM work
+ * pads the ragged non-local time.  The placement is solved on the host
+ * (section 6) and filled once (Filler).
+ *
+ * Conventions that hold for every function:
+ *  - Errors: every function returns a ugache_status; nothing throws or aborts across the
+ *    ABI.  UGACHE_EINVAL = bad argument / size / alignment; UGACHE_ESTATE = wrong call
+ *    order; UGACHE_ECUDA = a CUDA runtime call failed (text in ugache_last_error_message);
+ *    UGACHE_ENOMEM = device or host allocation failed; UGACHE_EPEER = peer mapping failed.
+ *  - Pointers are plain host or device addresses.  Streams are cudaStream_t passed as
+ *    void* (NULL = legacy default stream).
+ *  - Keys are integer row ids in [0, num_rows).  An out-of-range key (including a negative
+ *    int64) yields an all-zero output row and is counted in bad_keys (R2).
+ *  - Sizes: num_rows < 2^32, batch n < 2^32, row_bytes a positive multiple of 16.
+ *  - One ugache_ctx per (process, GPU rank).  A ctx is not re-entrant: calls on one ctx
+ *    must not overlap; extracts on one ctx are ordered by the caller's streams.
+ */
+#ifndef UGACHE_H_
+#define UGACHE_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define UGACHE_VERSION 1
+#define UGACHE_MAX_GPUS 16
+/* Location-table entry: (src << 56) | row.  src = j < G: GPU j's cache slab, row = slot;
+ * src = G: host DRAM, row = key (the host holds every entry). */
+#define UGACHE_LOC_SRC_SHIFT 56
+#define UGACHE_LOC_ROW_MASK ((((uint64_t)1) << 56) - 1)
+
+typedef struct ugache_ctx ugache_ctx;
+
+typedef enum {
+  UGACHE_OK = 0,
+  UGACHE_EINVAL = 1,
+  UGACHE_ECUDA = 2,
+  UGACHE_ENOMEM = 3,
+  UGACHE_ESTATE = 4,
+  UGACHE_EPEER = 5,
+  UGACHE_EKEY = 6
+} ugache_status;
+
+/* Cache policies run through the same kernels (P:385-413 replication / partition;
+ * UGACHE = hotness-driven hot-replicate / warm-partition chosen by the section 6.2 model). */
+typedef enum {
+  UGACHE_POLICY_UGACHE = 0,
+  UGACHE_POLICY_REPLICATION = 1,
+  UGACHE_POLICY_PARTITION = 2
+} ugache_policy;
+
+typedef enum { UGACHE_KEY_I64 = 0, UGACHE_KEY_U32 = 1 } ugache_key_type;
+
+/* Extraction mechanism.  FACTORED = the paper's FEM (section 5.3).  RANDOM_DISPATCH = the
+ * unfactored peer-based baseline (section 5.2): keys dispatched to warps in
+ * input order, each warp locates on the fly and reads whichever source (ablation only). */
+typedef enum { UGACHE_MODE_FACTORED = 0, UGACHE_MODE_RANDOM_DISPATCH = 1 } ugache_mode;
+
+typedef struct {
+  uint64_t num_rows;      /* N: entries of the (concatenated) embedding table            */
+  uint32_t row_bytes;     /* R: bytes per entry (D * sizeof(dtype)), multiple of 16       */
+  uint32_t reserved0;     /* must be 0                                                    */
+  uint64_t capacity_rows; /* C: per-GPU cache capacity in entries (Cap_j) */
+  int32_t num_gpus;       /* G in [1, UGACHE_MAX_GPUS]                                    */
+  int32_t rank;           /* this GPU's index in [0, G)                                   */
+  int32_t device;         /* CUDA device ordinal used by this ctx                         */
+  int32_t policy;         /* ugache_policy                                                */
+  double bw_local;        /* bytes/s of local HBM gathers for the model; 0 = default      */
+  double bw_peer;         /* bytes/s of NVLink ingress per GPU; 0 = default               */
+  double bw_host;         /* bytes/s of host->GPU zero-copy reads; 0 = default            */
+  int32_t host_sms;       /* SMs dedicated to host extraction; 0 = default  */
+  int32_t peer_sms;       /* SMs dedicated to each peer; 0 = floor((S-host)/(G-1)) */
+  int32_t num_sms;        /* S; 0 = the device's SM count (148 on B200)                   */
+  int32_t flags;          /* must be 0                                                    */
+} ugache_config;
+
+/* Solver output (section 6.2 model evaluated for the chosen placement). */
+typedef struct {
+  int32_t policy;          /* policy solved for                                         */
+  int32_t num_gpus;        /* G                                                         */
+  uint64_t capacity_rows;  /* effective C = min(C, N)                                   */
+  uint64_t k;              /* hotness ranks [0,k) replicated on every GPU               */
+  uint64_t band_end;       /* ranks [k,band_end) partitioned round-robin; rest on host  */
+  double z;                /* modeled batch extraction time (s) of the chosen placement */
+  double z_replication;    /* z at k = C                                                */
+  double z_partition;      /* z at k = 0                                                */
+  double T_local, T_peer, T_host;  /* T_{i<-j} per entry (s)               */
+  double R_local, R_peer, R_host;  /* R_{i<-j} core ratios                   */
+  int32_t host_sms, peer_sms, num_sms, reserved;
+} ugache_plan;
+
+/* ---- host-only placement solver (no GPU needed) ------------------------------------ */
+
+/* Solve the cache placement (section 6) for cfg (rank/device ignored).
+ * hotness: N floats (access frequency; NULL = uniform; NaN/Inf -> EINVAL;
+ * values <= 0 count as 0).  order: optional out, N entries, order[r] = key of hotness rank
+ * r (ties by lower key).  plan: out.  Deterministic; O(N) memory + O(C*G) model sweep. */
+ugache_status ugache_solve(const ugache_config *cfg, const float *hotness, uint64_t *order,
+                           ugache_plan *plan);
+
+/* Build GPU `gpu`'s location table and slot list for a solved plan.
+ * order: N entries from ugache_solve.  loc: out, N entries (UGACHE_LOC_* encoding).
+ * slot_keys: out, capacity_rows entries (key cached in each slot of GPU gpu's slab);
+ * n_slots: out, number of filled slots (<= capacity). */
+ugache_status ugache_build_placement(const ugache_config *cfg, const uint64_t *order,
+                                     const ugache_plan *plan, int32_t gpu, uint64_t *loc,
+                                     uint64_t *slot_keys, uint64_t *n_slots);
+
+/* ---- context lifecycle -------------------------------------------------------------- */
+
+/* Create the ctx of GPU cfg->rank on device cfg->device: solve the placement, build this
+ * GPU's location table in HBM, allocate the cache slab (C x R bytes, its own cudaMalloc so
+ * it can be IPC-exported) and the bucket scratch.  host_table: N*R bytes, caller-owned, must
+ * outlive the ctx and stay unmodified (read-only access); it is page-locked and
+ * mapped with cudaHostRegister unless already pinned.  hotness: as for ugache_solve,
+ * copied.  The cache is NOT filled: call ugache_fill, connect peers, then barrier. */
+ugache_status ugache_init(ugache_ctx **ctx, const ugache_config *cfg, const void *host_table,
+                          const float *hotness);
+
+/* Same as ugache_init but with a precomputed order/plan (every rank of a process group can
+ * share one solve).  order: N entries; plan from ugache_solve with the same cfg. */
+ugache_status ugache_init_with_plan(ugache_ctx **ctx, const ugache_config *cfg,
+                                    const void *host_table, const uint64_t *order,
+                                    const ugache_plan *plan);
+
+ugache_status ugache_get_plan(const ugache_ctx *ctx, ugache_plan *plan);
+
+/* Device address and size of this GPU's cache slab (for in-process peers / checks). */
+ugache_status ugache_slab(const ugache_ctx *ctx, void **dev_ptr, uint64_t *bytes,
+                          uint64_t *n_slots);
+
+/* Export this GPU's slab as a cudaIpcMemHandle_t.  buf: out, *len in: capacity, out: bytes
+ * written (64).  Peer-based access in a unified address space. */
+ugache_status ugache_ipc_handle(ugache_ctx *ctx, void *buf, size_t *len);
+
+/* Map every peer's slab.  all_handles: G handles of len_each bytes in rank order (this
+ * rank's entry is ignored).  Opened with cudaIpcMemLazyEnablePeerAccess.  -> EPEER. */
+ugache_status ugache_open_peers(ugache_ctx *ctx, const void *all_handles, size_t len_each);
+
+/* In-process alternative to IPC: slabs[j] = device address of GPU j's slab, reachable from
+ * this ctx's device (same device, or peer access enabled).  slabs[rank] is ignored. */
+ugache_status ugache_set_peer_slabs(ugache_ctx *ctx, const void *const *slabs);
+
+/* Filler: copy this GPU's cached rows from the host table into its slab
+ * (zero-copy gather over PCIe), asynchronously on stream.  Peers must be filled (and a
+ * barrier passed) before any GPU extracts from them. */
+ugache_status ugache_fill(ugache_ctx *ctx, void *stream);
+
+/* THE HOT PATH.  out[i*R .. (i+1)*R) = table row keys[i] for i < n (output in
+ * key order P:626-627).  keys: n keys of key_type, device or host memory.  out: n*R bytes,
+ * device or host memory, 16-byte aligned.  Device buffers: fully asynchronous on stream,
+ * no host synchronisation, no collective; keys/out must stay valid until the stream
+ * reaches the work.  Host buffers: staged through ctx-owned device buffers with async
+ * copies on the same stream (the caller synchronises the stream before reading out).
+ * n == 0: no work.  Requires ugache_fill and, for G > 1, peers (else ESTATE). */
+ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type, uint64_t n,
+                             void *out, void *stream);
+
+/* Core dedication override: SMs for host and for each peer; local gets the
+ * rest plus padding.  0 keeps the current value.  Only affects later extracts. */
+ugache_status ugache_set_dedication(ugache_ctx *ctx, int32_t host_sms, int32_t peer_sms);
+
+/* ugache_mode; FACTORED by default. */
+ugache_status ugache_set_mode(ugache_ctx *ctx, int32_t mode);
+
+/* Per-source key counts of the last extract: per_source[j] for GPU j (j == rank: local),
+ * per_source[G] for host (G+1 entries); bad_keys: out-of-range keys.  Synchronises with
+ * the last extract.  Per-source hit rates as in Fig. 14. */
+ugache_status ugache_last_batch_stats(ugache_ctx *ctx, uint64_t *per_source,
+                                      uint64_t *bad_keys);
+
+/* When enabled, extract records CUDA events around its locate+bucket and gather kernels on
+ * the extract stream; ugache_last_batch_timing synchronises and returns their durations. */
+ugache_status ugache_enable_timing(ugache_ctx *ctx, int32_t on);
+ugache_status ugache_last_batch_timing(ugache_ctx *ctx, float *ms_locate, float *ms_gather);
+
+/* Number of kernel launches the last extract issued (for launch accounting). */
+ugache_status ugache_last_launch_count(const ugache_ctx *ctx, int32_t *launches);
+
+/* Copy out this GPU's location table (N entries) and slot list (capacity entries) for the
+ * placement checker.  Synchronous. */
+ugache_status ugache_export_placement(ugache_ctx *ctx, uint64_t *loc, uint64_t *slot_keys,
+                                      uint64_t *n_slots);
+
+/* Copy slots [first, first+count) of this GPU's slab to host memory dst (count*R bytes). */
+ugache_status ugache_read_slab(ugache_ctx *ctx, uint64_t first, uint64_t count, void *dst);
+
+/* Release device memory, peer mappings and the host-table registration. NULL is a no-op. */
+ugache_status ugache_destroy(ugache_ctx *ctx);
+
+const char *ugache_error_string(ugache_status st);
+const char *ugache_last_error_message(const ugache_ctx *ctx);
+int32_t ugache_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* UGACHE_H_ */

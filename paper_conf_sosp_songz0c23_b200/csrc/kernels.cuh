@@ -1,0 +1,360 @@
+// kernels.cuh -- sm_100a kernels of the factored extraction path.
+//
+//  K1 locate_bucket_kernel : key -> location-table entry -> per-source bucket
+//                            (locate; grouping)
+//  K2 factored_gather_kernel : one CTA per SM, CTA role = source; non-local roles copy
+//                            their bucket first, then every CTA pads the local bucket
+//                            through an atomic cursor (FEM)
+//  K2' random_dispatch_kernel : unfactored peer-based baseline, ablation only
+//  K5 fill_kernel          : Filler, host rows -> this GPU's cache slab
+//
+// Nothing here is a contraction: every step is integer address arithmetic plus 16-byte
+// vector copies, so the kernels are written for HBM / NVLink / PCIe bandwidth (coalesced
+// 16-B lanes, many independent rows in flight per warp, streaming store hints).
+#pragma once
+
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "ugache.h"
+
+namespace ugk {
+
+constexpr int kMaxSrc = UGACHE_MAX_GPUS + 1;
+constexpr int kLocateThreads = 256;
+constexpr int kLocateItems = 8;  // keys per thread -> 2048-key tile per CTA
+constexpr int kLocateTile = kLocateThreads * kLocateItems;
+constexpr int kGatherThreads = 512;  // 16 warps; one CTA per SM (forced via smem)
+constexpr int kGatherWarps = kGatherThreads / 32;
+constexpr int kRowsInFlight = 8;     // rows per warp per step (U)
+constexpr int kLocalChunk = 64;      // rows per local-cursor claim
+constexpr uint32_t kFullMask = 0xFFFFFFFFu;
+
+// Device control block (one per ctx).  counts/local_cursor/done/bad are consumed and reset
+// by the last CTA of every gather launch, so consecutive extracts need no memset.
+struct Ctrl {
+  uint32_t counts[kMaxSrc];
+  uint32_t local_cursor;
+  uint32_t done;
+  uint32_t bad;
+  uint32_t stat_counts[kMaxSrc];
+  uint32_t stat_bad;
+  uint32_t pad[4];
+};
+
+struct LocateParams {
+  const void *keys;
+  const uint64_t *loc;       // N entries, (src << 56) | row
+  uint64_t *buckets;         // num_src x bucket_cap entries, (row << 32) | out_idx
+  Ctrl *ctrl;
+  uint8_t *out;              // for zero rows of out-of-range keys
+  uint64_t num_rows;
+  uint64_t bucket_cap;
+  uint32_t n;
+  uint32_t row_bytes;
+  int32_t num_src;
+};
+
+struct GatherParams {
+  const uint64_t *buckets;
+  Ctrl *ctrl;
+  const uint8_t *base[kMaxSrc];  // row base address of each source
+  uint8_t *out;
+  uint64_t bucket_cap;
+  uint32_t row_bytes;
+  int32_t num_src;
+  int32_t local_src;
+  int32_t n_roles;
+  int32_t role_src[kMaxSrc];       // role r serves source role_src[r]
+  int32_t role_cta_end[kMaxSrc];   // CTAs [role_cta_end[r-1], role_cta_end[r]) have role r
+};
+
+struct RandomParams {
+  const void *keys;
+  const uint64_t *loc;
+  Ctrl *ctrl;
+  const uint8_t *base[kMaxSrc];
+  uint8_t *out;
+  uint64_t num_rows;
+  uint32_t n;
+  uint32_t row_bytes;
+  int32_t num_src;
+};
+
+struct FillParams {
+  const uint64_t *slot_keys;
+  const uint8_t *table;  // device-mapped host table
+  uint8_t *slab;
+  uint64_t n_slots;
+  uint32_t row_bytes;
+};
+
+// ---------------------------------------------------------------------------- helpers
+__device__ __forceinline__ uint4 ld_nc_v4(const void *p) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+__device__ __forceinline__ void st_cs_v4(void *p, const uint4 &v) {
+  asm volatile("st.global.cs.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y),
+               "r"(v.z), "r"(v.w)
+               : "memory");
+}
+__device__ __forceinline__ uint64_t ld_nc_u64(const uint64_t *p) {
+  uint64_t r;
+  asm volatile("ld.global.nc.u64 %0, [%1];" : "=l"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
+// Warp copies up to U rows.  ent: bucket entries (row << 32 | out_idx), read by lanes < U.
+// All U loads of a lane are issued before its stores (U * 16 B in flight per lane per
+// vector step).  Rows of R bytes = V 16-byte vectors; lanes stride over V.
+template <int U>
+__device__ __forceinline__ void copy_rows(const uint8_t *__restrict__ base,
+                                          uint8_t *__restrict__ out, uint32_t R,
+                                          const uint64_t *__restrict__ ent, int nvalid,
+                                          int lane) {
+  const uint64_t e = (lane < nvalid) ? ent[lane] : 0ull;
+  uint64_t eu[U];
+#pragma unroll
+  for (int u = 0; u < U; ++u) eu[u] = __shfl_sync(kFullMask, e, u);
+  const uint32_t V = R >> 4;
+  for (uint32_t j = lane; j < V; j += 32) {
+    uint4 v[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (u < nvalid) v[u] = ld_nc_v4(base + (eu[u] >> 32) * (uint64_t)R + (uint64_t)j * 16u);
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (u < nvalid)
+        st_cs_v4(out + (eu[u] & 0xFFFFFFFFull) * (uint64_t)R + (uint64_t)j * 16u, v[u]);
+  }
+}
+
+__device__ __forceinline__ void zero_row(uint8_t *dst, uint32_t R) {
+  const uint4 z = make_uint4(0, 0, 0, 0);
+  for (uint32_t j = 0; j < (R >> 4); ++j) *reinterpret_cast<uint4 *>(dst + (uint64_t)j * 16) = z;
+}
+
+template <typename KeyT>
+__device__ __forceinline__ bool key_in_range(KeyT k, uint64_t N) {
+  if constexpr (sizeof(KeyT) == 8) return k >= 0 && (uint64_t)k < N;
+  else return (uint64_t)k < N;
+}
+
+// Last CTA of a gather launch publishes stats and re-arms the control block.
+__device__ __forceinline__ void finish_launch(Ctrl *ctrl, int num_src) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const uint32_t prev = atomicAdd(&ctrl->done, 1u);
+    if (prev == gridDim.x - 1) {
+      __threadfence();
+      volatile Ctrl *c = ctrl;
+      for (int s = 0; s < num_src; ++s) {
+        c->stat_counts[s] = c->counts[s];
+        c->counts[s] = 0;
+      }
+      c->stat_bad = c->bad;
+      c->bad = 0;
+      c->local_cursor = 0;
+      __threadfence();
+      c->done = 0;
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------- K1
+template <typename KeyT>
+__global__ void __launch_bounds__(kLocateThreads)
+    locate_bucket_kernel(const LocateParams p) {
+  __shared__ uint32_t s_cnt[kMaxSrc];
+  __shared__ uint32_t s_base[kMaxSrc];
+  const int tid = threadIdx.x, lane = tid & 31;
+  if (tid < kMaxSrc) s_cnt[tid] = 0;
+  __syncthreads();
+  const KeyT *keys = static_cast<const KeyT *>(p.keys);
+  const uint64_t tile0 = (uint64_t)blockIdx.x * kLocateTile;
+
+  KeyT k[kLocateItems];
+  uint64_t e[kLocateItems];
+#pragma unroll
+  for (int it = 0; it < kLocateItems; ++it) {  // coalesced key loads
+    const uint64_t i = tile0 + (uint64_t)it * kLocateThreads + tid;
+    k[it] = (i < p.n) ? keys[i] : (KeyT)0;
+  }
+#pragma unroll
+  for (int it = 0; it < kLocateItems; ++it) {  // random location-table reads, all in flight
+    const uint64_t i = tile0 + (uint64_t)it * kLocateThreads + tid;
+    e[it] = (i < p.n && key_in_range<KeyT>(k[it], p.num_rows)) ? ld_nc_u64(p.loc + (uint64_t)k[it])
+                                                               : ~0ull;
+  }
+  int src[kLocateItems];
+  uint32_t pos[kLocateItems];
+  uint32_t nbad = 0;
+#pragma unroll
+  for (int it = 0; it < kLocateItems; ++it) {
+    const uint64_t i = tile0 + (uint64_t)it * kLocateThreads + tid;
+    int s = -1;
+    if (i < p.n) {
+      if (e[it] != ~0ull) {
+        s = (int)(e[it] >> UGACHE_LOC_SRC_SHIFT);
+      } else {
+        zero_row(p.out + i * (uint64_t)p.row_bytes, p.row_bytes);  // out-of-range key
+        ++nbad;
+      }
+    }
+    // warp-aggregated per-source slot reservation in shared memory
+    const uint32_t peers = __match_any_sync(kFullMask, s);
+    const int leader = __ffs(peers) - 1;
+    uint32_t b = 0;
+    if (s >= 0 && lane == leader) b = atomicAdd(&s_cnt[s], (uint32_t)__popc(peers));
+    b = __shfl_sync(kFullMask, b, leader);
+    src[it] = s;
+    pos[it] = b + __popc(peers & lanemask_lt());
+  }
+  if (nbad) atomicAdd(&p.ctrl->bad, nbad);
+  __syncthreads();
+  if (tid < p.num_src && s_cnt[tid]) s_base[tid] = atomicAdd(&p.ctrl->counts[tid], s_cnt[tid]);
+  __syncthreads();
+#pragma unroll
+  for (int it = 0; it < kLocateItems; ++it) {
+    if (src[it] >= 0) {
+      const uint64_t i = tile0 + (uint64_t)it * kLocateThreads + tid;
+      const uint32_t row = (uint32_t)(e[it] & UGACHE_LOC_ROW_MASK);
+      p.buckets[(uint64_t)src[it] * p.bucket_cap + s_base[src[it]] + pos[it]] =
+          ((uint64_t)row << 32) | (uint64_t)i;
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------- K2
+__global__ void __launch_bounds__(kGatherThreads, 1)
+    factored_gather_kernel(const GatherParams p) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  int r = 0;
+  while (r < p.n_roles - 1 && (int)blockIdx.x >= p.role_cta_end[r]) ++r;
+  const int my_src = p.role_src[r];
+  const int cta_begin = r ? p.role_cta_end[r - 1] : 0;
+  const int role_ctas = p.role_cta_end[r] - cta_begin;
+  const uint32_t R = p.row_bytes;
+
+  if (my_src != p.local_src) {
+    // dedicated non-local extraction: static warp striding over this source's bucket
+    const uint32_t cnt = p.ctrl->counts[my_src];
+    const uint64_t *b = p.buckets + (uint64_t)my_src * p.bucket_cap;
+    const uint8_t *base = p.base[my_src];
+    const uint32_t W = (uint32_t)role_ctas * kGatherWarps;
+    const uint32_t gw = (uint32_t)((int)blockIdx.x - cta_begin) * kGatherWarps + warp;
+    for (uint32_t e0 = gw * kRowsInFlight; e0 < cnt; e0 += W * kRowsInFlight)
+      copy_rows<kRowsInFlight>(base, p.out, R, b + e0, (int)min((uint32_t)kRowsInFlight, cnt - e0),
+                               lane);
+  }
+  // local group: dedicated local CTAs start here; others pad once their group drains
+  {
+    const uint32_t cnt = p.ctrl->counts[p.local_src];
+    const uint64_t *b = p.buckets + (uint64_t)p.local_src * p.bucket_cap;
+    const uint8_t *base = p.base[p.local_src];
+    uint32_t next = 0;
+    if (lane == 0) next = atomicAdd(&p.ctrl->local_cursor, (uint32_t)kLocalChunk);
+    next = __shfl_sync(kFullMask, next, 0);
+    while (next < cnt) {
+      const uint32_t c0 = next, c1 = min(cnt, c0 + (uint32_t)kLocalChunk);
+      if (lane == 0) next = atomicAdd(&p.ctrl->local_cursor, (uint32_t)kLocalChunk);  // prefetch claim
+      next = __shfl_sync(kFullMask, next, 0);
+      for (uint32_t e0 = c0; e0 < c1; e0 += kRowsInFlight)
+        copy_rows<kRowsInFlight>(base, p.out, R, b + e0, (int)min((uint32_t)kRowsInFlight, c1 - e0),
+                                 lane);
+    }
+  }
+  finish_launch(p.ctrl, p.num_src);
+}
+
+// ---------------------------------------------------------------------------- K2'
+template <typename KeyT>
+__global__ void __launch_bounds__(kGatherThreads, 1)
+    random_dispatch_kernel(const RandomParams p) {
+  __shared__ uint32_t s_cnt[kMaxSrc];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x < kMaxSrc) s_cnt[threadIdx.x] = 0;
+  __syncthreads();
+  const KeyT *keys = static_cast<const KeyT *>(p.keys);
+  const uint32_t R = p.row_bytes, V = R >> 4;
+  const uint32_t W = gridDim.x * kGatherWarps;
+  uint32_t nbad = 0;
+  for (uint32_t e0 = (blockIdx.x * kGatherWarps + warp) * kRowsInFlight; e0 < p.n;
+       e0 += W * kRowsInFlight) {
+    const int nvalid = (int)min((uint32_t)kRowsInFlight, p.n - e0);
+    int s = -2;
+    uint64_t rr = 0;
+    if (lane < nvalid) {
+      const KeyT k = keys[e0 + lane];
+      if (key_in_range<KeyT>(k, p.num_rows)) {
+        const uint64_t e = ld_nc_u64(p.loc + (uint64_t)k);
+        s = (int)(e >> UGACHE_LOC_SRC_SHIFT);
+        rr = e & UGACHE_LOC_ROW_MASK;
+      } else {
+        s = -1;
+        ++nbad;
+      }
+    }
+    const uint32_t peers = __match_any_sync(kFullMask, s);
+    if (s >= 0 && lane == __ffs(peers) - 1) atomicAdd(&s_cnt[s], (uint32_t)__popc(peers));
+    int su[kRowsInFlight];
+    uint64_t ru[kRowsInFlight];
+#pragma unroll
+    for (int u = 0; u < kRowsInFlight; ++u) {
+      su[u] = __shfl_sync(kFullMask, s, u);
+      ru[u] = __shfl_sync(kFullMask, rr, u);
+    }
+    for (uint32_t j = lane; j < V; j += 32) {
+      uint4 v[kRowsInFlight];
+#pragma unroll
+      for (int u = 0; u < kRowsInFlight; ++u)
+        if (su[u] >= 0) v[u] = ld_nc_v4(p.base[su[u]] + ru[u] * R + (uint64_t)j * 16u);
+        else v[u] = make_uint4(0, 0, 0, 0);
+#pragma unroll
+      for (int u = 0; u < kRowsInFlight; ++u)
+        if (su[u] >= -1) st_cs_v4(p.out + (uint64_t)(e0 + u) * R + (uint64_t)j * 16u, v[u]);
+    }
+  }
+  if (nbad) atomicAdd(&p.ctrl->bad, nbad);
+  __syncthreads();
+  if (threadIdx.x < p.num_src && s_cnt[threadIdx.x])
+    atomicAdd(&p.ctrl->counts[threadIdx.x], s_cnt[threadIdx.x]);
+  finish_launch(p.ctrl, p.num_src);
+}
+
+// ---------------------------------------------------------------------------- K5
+__global__ void __launch_bounds__(256) fill_kernel(const FillParams p) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t W = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  const uint32_t V = p.row_bytes >> 4;
+  for (uint64_t s0 = warp * kRowsInFlight; s0 < p.n_slots; s0 += W * kRowsInFlight) {
+    const int nvalid = (int)min((uint64_t)kRowsInFlight, p.n_slots - s0);
+    const uint64_t key = lane < nvalid ? p.slot_keys[s0 + lane] : 0ull;
+    uint64_t ku[kRowsInFlight];
+#pragma unroll
+    for (int u = 0; u < kRowsInFlight; ++u) ku[u] = __shfl_sync(kFullMask, key, u);
+    for (uint32_t j = lane; j < V; j += 32) {
+      uint4 v[kRowsInFlight];
+#pragma unroll
+      for (int u = 0; u < kRowsInFlight; ++u)
+        if (u < nvalid) v[u] = ld_nc_v4(p.table + ku[u] * p.row_bytes + (uint64_t)j * 16u);
+#pragma unroll
+      for (int u = 0; u < kRowsInFlight; ++u)
+        if (u < nvalid)
+          *reinterpret_cast<uint4 *>(p.slab + (s0 + u) * p.row_bytes + (uint64_t)j * 16u) = v[u];
+    }
+  }
+}
+
+}  // namespace ugk

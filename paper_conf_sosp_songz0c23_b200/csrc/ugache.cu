@@ -1,0 +1,646 @@
+// ugache.cu -- C ABI of libugache: context, host-table mapping, peers, fill, extract.
+//
+// See include/ugache.h for the contract of every entry point.  The per-batch path is
+// ugache_extract -> K1 locate_bucket_kernel -> K2 factored_gather_kernel (kernels.cuh),
+// two launches on the caller's stream with no host synchronisation and no collective.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "kernels.cuh"
+#include "ugache_internal.h"
+
+struct ugache_ctx {
+  ugache_config cfg{};
+  ugache_plan plan{};
+  int device = 0;
+  int sm_count = 0;
+  // host table (source G)
+  const uint8_t *host_table = nullptr;
+  const uint8_t *host_table_dev = nullptr;
+  bool registered = false;
+  // this GPU's cache slab and location table
+  uint8_t *slab = nullptr;
+  uint64_t slab_bytes = 0;
+  uint64_t n_slots = 0;
+  uint64_t *d_slot_keys = nullptr;
+  uint64_t *d_loc = nullptr;
+  // sources
+  const uint8_t *src_base[ug::kMaxSrc] = {};
+  void *ipc_mapped[UGACHE_MAX_GPUS] = {};
+  bool peers_ready = false;
+  bool filled = false;
+  // scratch
+  ugk::Ctrl *d_ctrl = nullptr;
+  uint64_t *d_buckets = nullptr;
+  uint64_t bucket_cap = 0;
+  void *d_keys_stage = nullptr;
+  size_t keys_stage_bytes = 0;
+  void *d_out_stage = nullptr;
+  size_t out_stage_bytes = 0;
+  // dedication / mode
+  int host_sms = 0, peer_sms = 0;
+  int mode = UGACHE_MODE_FACTORED;
+  // timing
+  bool timing = false;
+  bool timing_valid = false;
+  cudaEvent_t ev[3] = {};
+  int last_launches = 0;
+  uint64_t last_n = 0;
+  cudaStream_t last_stream = nullptr;
+  std::string err;
+};
+
+namespace {
+
+// Dynamic shared memory requested only to guarantee one gather CTA per SM, so that the
+// CTA index -> role mapping is also an SM -> role mapping (P:1620-1627 used MPS for this).
+constexpr size_t kOneCtaPerSmSmem = 120 * 1024;
+
+std::mutex g_reg_mu;
+std::map<const void *, int> g_reg_count;  // host-table registrations owned by this library
+
+ugache_status cuda_fail(ugache_ctx *ctx, cudaError_t e, const char *what) {
+  if (ctx) {
+    char buf[512];
+    snprintf(buf, sizeof(buf), "%s: %s (%s)", what, cudaGetErrorName(e), cudaGetErrorString(e));
+    ctx->err = buf;
+  }
+  (void)cudaGetLastError();
+  return e == cudaErrorMemoryAllocation ? UGACHE_ENOMEM : UGACHE_ECUDA;
+}
+
+#define UG_CUDA(ctx, call)                                  \
+  do {                                                      \
+    cudaError_t _e = (call);                                \
+    if (_e != cudaSuccess) return cuda_fail(ctx, _e, #call); \
+  } while (0)
+
+ugache_status fail(ugache_ctx *ctx, ugache_status st, const char *msg) {
+  if (ctx) ctx->err = msg;
+  return st;
+}
+
+bool is_device_pointer(const void *p, int *device) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    (void)cudaGetLastError();
+    return false;
+  }
+  if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) {
+    if (device) *device = a.device;
+    return true;
+  }
+  return false;
+}
+
+bool is_pinned_host(const void *p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    (void)cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeHost;
+}
+
+ugache_status register_host_table(ugache_ctx *ctx, const void *table, size_t bytes) {
+  std::lock_guard<std::mutex> lk(g_reg_mu);
+  auto it = g_reg_count.find(table);
+  if (it != g_reg_count.end()) {
+    it->second++;
+    ctx->registered = true;
+  } else if (!is_pinned_host(table)) {
+    cudaError_t e = cudaHostRegister(const_cast<void *>(table), bytes,
+                                     cudaHostRegisterMapped | cudaHostRegisterPortable |
+                                         cudaHostRegisterReadOnly);
+    if (e != cudaSuccess) {
+      (void)cudaGetLastError();
+      e = cudaHostRegister(const_cast<void *>(table), bytes,
+                           cudaHostRegisterMapped | cudaHostRegisterPortable);
+    }
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "cudaHostRegister(host_table)");
+    g_reg_count[table] = 1;
+    ctx->registered = true;
+  }
+  void *dptr = nullptr;
+  UG_CUDA(ctx, cudaHostGetDevicePointer(&dptr, const_cast<void *>(table), 0));
+  ctx->host_table_dev = static_cast<const uint8_t *>(dptr);
+  return UGACHE_OK;
+}
+
+void unregister_host_table(ugache_ctx *ctx) {
+  if (!ctx->registered) return;
+  std::lock_guard<std::mutex> lk(g_reg_mu);
+  auto it = g_reg_count.find(ctx->host_table);
+  if (it != g_reg_count.end() && --it->second == 0) {
+    cudaHostUnregister(const_cast<uint8_t *>(ctx->host_table));
+    (void)cudaGetLastError();
+    g_reg_count.erase(it);
+  }
+  ctx->registered = false;
+}
+
+ugache_status ensure_scratch(ugache_ctx *ctx, uint64_t n) {
+  if (n <= ctx->bucket_cap) return UGACHE_OK;
+  uint64_t cap = std::max<uint64_t>(n, 1024);
+  if (ctx->d_buckets) {
+    UG_CUDA(ctx, cudaDeviceSynchronize());
+    cudaFree(ctx->d_buckets);
+    ctx->d_buckets = nullptr;
+    ctx->bucket_cap = 0;
+  }
+  const size_t bytes = (size_t)(ctx->cfg.num_gpus + 1) * cap * sizeof(uint64_t);
+  UG_CUDA(ctx, cudaMalloc(&ctx->d_buckets, bytes));
+  ctx->bucket_cap = cap;
+  return UGACHE_OK;
+}
+
+ugache_status ensure_stage(ugache_ctx *ctx, void **buf, size_t *have, size_t need) {
+  if (need <= *have) return UGACHE_OK;
+  if (*buf) {
+    UG_CUDA(ctx, cudaDeviceSynchronize());
+    cudaFree(*buf);
+    *buf = nullptr;
+    *have = 0;
+  }
+  UG_CUDA(ctx, cudaMalloc(buf, need));
+  *have = need;
+  return UGACHE_OK;
+}
+
+// Role table of the gather kernel: host first, then each peer, then local.
+void build_roles(const ugache_ctx *ctx, ugk::GatherParams *gp, int *grid) {
+  const int G = ctx->cfg.num_gpus, me = ctx->cfg.rank, S = ctx->sm_count;
+  int nr = 0, end = 0;
+  gp->role_src[nr] = G;  // host
+  end += ctx->host_sms;
+  gp->role_cta_end[nr++] = end;
+  for (int j = 0; j < G; ++j) {
+    if (j == me) continue;
+    gp->role_src[nr] = j;
+    end += ctx->peer_sms;
+    gp->role_cta_end[nr++] = end;
+  }
+  if (end < S) {
+    gp->role_src[nr] = me;
+    end = S;
+    gp->role_cta_end[nr++] = end;
+  }
+  gp->n_roles = nr;
+  *grid = end;
+}
+
+ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void *host_table,
+                          const std::vector<uint32_t> &order) {
+  const uint64_t N = cfg->num_rows, R = cfg->row_bytes;
+  const int G = cfg->num_gpus;
+  ugache_status st = register_host_table(ctx, host_table, (size_t)(N * R));
+  if (st != UGACHE_OK) return st;
+  ctx->host_table = static_cast<const uint8_t *>(host_table);
+
+  // location table and slot list of this rank
+  std::vector<uint64_t> loc;
+  std::vector<uint64_t> slots;
+  try {
+    loc.resize(N);
+    slots.resize(std::max<uint64_t>(ctx->plan.capacity_rows, 1));
+  } catch (const std::bad_alloc &) {
+    return fail(ctx, UGACHE_ENOMEM, "host allocation of the location table failed");
+  }
+  st = ug::build_placement(cfg, order.data(), &ctx->plan, cfg->rank, loc.data(), slots.data(),
+                           &ctx->n_slots);
+  if (st != UGACHE_OK) return fail(ctx, st, "build_placement failed");
+
+  ctx->slab_bytes = std::max<uint64_t>(ctx->plan.capacity_rows, 1) * R;
+  UG_CUDA(ctx, cudaMalloc(&ctx->slab, ctx->slab_bytes));
+  UG_CUDA(ctx, cudaMalloc(&ctx->d_loc, N * sizeof(uint64_t)));
+  UG_CUDA(ctx, cudaMemcpy(ctx->d_loc, loc.data(), N * sizeof(uint64_t), cudaMemcpyHostToDevice));
+  if (ctx->n_slots) {
+    UG_CUDA(ctx, cudaMalloc(&ctx->d_slot_keys, ctx->n_slots * sizeof(uint64_t)));
+    UG_CUDA(ctx, cudaMemcpy(ctx->d_slot_keys, slots.data(), ctx->n_slots * sizeof(uint64_t),
+                            cudaMemcpyHostToDevice));
+  }
+  UG_CUDA(ctx, cudaMalloc(&ctx->d_ctrl, sizeof(ugk::Ctrl)));
+  UG_CUDA(ctx, cudaMemset(ctx->d_ctrl, 0, sizeof(ugk::Ctrl)));
+  for (int i = 0; i < 3; ++i) UG_CUDA(ctx, cudaEventCreate(&ctx->ev[i]));
+  ctx->src_base[cfg->rank] = ctx->slab;
+  ctx->src_base[G] = ctx->host_table_dev;
+  ctx->peers_ready = (G == 1);
+  ctx->host_sms = ctx->plan.host_sms;
+  ctx->peer_sms = ctx->plan.peer_sms;
+  UG_CUDA(ctx, cudaFuncSetAttribute(ugk::factored_gather_kernel,
+                                    cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem));
+  UG_CUDA(ctx, cudaFuncSetAttribute(ugk::random_dispatch_kernel<int64_t>,
+                                    cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem));
+  UG_CUDA(ctx, cudaFuncSetAttribute(ugk::random_dispatch_kernel<uint32_t>,
+                                    cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem));
+  return UGACHE_OK;
+}
+
+ugache_status begin(ugache_ctx *ctx) {
+  UG_CUDA(ctx, cudaSetDevice(ctx->device));
+  return UGACHE_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int32_t ugache_version(void) { return UGACHE_VERSION; }
+
+const char *ugache_error_string(ugache_status st) {
+  switch (st) {
+    case UGACHE_OK: return "ok";
+    case UGACHE_EINVAL: return "invalid argument";
+    case UGACHE_ECUDA: return "CUDA error";
+    case UGACHE_ENOMEM: return "out of memory";
+    case UGACHE_ESTATE: return "invalid call order";
+    case UGACHE_EPEER: return "peer mapping failed";
+    case UGACHE_EKEY: return "key out of range";
+  }
+  return "unknown status";
+}
+
+const char *ugache_last_error_message(const ugache_ctx *ctx) {
+  return ctx ? ctx->err.c_str() : "";
+}
+
+static ugache_status init_impl(ugache_ctx **out, const ugache_config *cfg, const void *host_table,
+                               const float *hotness, const uint64_t *order_in,
+                               const ugache_plan *plan_in) {
+  if (!out || !cfg || !host_table) return UGACHE_EINVAL;
+  *out = nullptr;
+  if (cfg->rank < 0 || cfg->rank >= cfg->num_gpus) return UGACHE_EINVAL;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= 0) {
+    (void)cudaGetLastError();
+    return UGACHE_ECUDA;
+  }
+  if (cfg->device < 0 || cfg->device >= ndev) return UGACHE_EINVAL;
+  ugache_ctx *ctx = new (std::nothrow) ugache_ctx();
+  if (!ctx) return UGACHE_ENOMEM;
+  ctx->cfg = *cfg;
+  ctx->device = cfg->device;
+  ugache_status st = begin(ctx);
+  if (st == UGACHE_OK) {
+    cudaError_t e = cudaDeviceGetAttribute(&ctx->sm_count, cudaDevAttrMultiProcessorCount, ctx->device);
+    if (e != cudaSuccess) st = cuda_fail(ctx, e, "cudaDeviceGetAttribute");
+  }
+  std::vector<uint32_t> order;
+  if (st == UGACHE_OK) {
+    if (order_in && plan_in) {
+      ug::Params p;
+      st = ug::resolve_params(cfg, ctx->sm_count, &p);
+      if (st == UGACHE_OK) {
+        order.resize(cfg->num_rows);
+        for (uint64_t i = 0; i < cfg->num_rows; ++i) {
+          if (order_in[i] >= cfg->num_rows) { st = UGACHE_EINVAL; break; }
+          order[i] = (uint32_t)order_in[i];
+        }
+        ctx->plan = *plan_in;
+        if (plan_in->num_gpus != cfg->num_gpus || plan_in->host_sms != p.host_sms ||
+            plan_in->peer_sms != p.peer_sms)
+          st = UGACHE_EINVAL;
+        if (plan_in->num_sms > ctx->sm_count) st = UGACHE_EINVAL;
+      }
+    } else {
+      st = ug::solve(cfg, ctx->sm_count, hotness, order, &ctx->plan);
+    }
+    if (st == UGACHE_OK && ctx->plan.num_sms > ctx->sm_count) st = UGACHE_EINVAL;
+  }
+  if (st == UGACHE_OK) st = init_common(ctx, cfg, host_table, order);
+  if (st != UGACHE_OK) {
+    ugache_destroy(ctx);
+    return st;
+  }
+  *out = ctx;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_init(ugache_ctx **ctx, const ugache_config *cfg, const void *host_table,
+                          const float *hotness) {
+  return init_impl(ctx, cfg, host_table, hotness, nullptr, nullptr);
+}
+
+ugache_status ugache_init_with_plan(ugache_ctx **ctx, const ugache_config *cfg,
+                                    const void *host_table, const uint64_t *order,
+                                    const ugache_plan *plan) {
+  if (!order || !plan) return UGACHE_EINVAL;
+  return init_impl(ctx, cfg, host_table, nullptr, order, plan);
+}
+
+ugache_status ugache_get_plan(const ugache_ctx *ctx, ugache_plan *plan) {
+  if (!ctx || !plan) return UGACHE_EINVAL;
+  *plan = ctx->plan;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_slab(const ugache_ctx *ctx, void **dev_ptr, uint64_t *bytes, uint64_t *n_slots) {
+  if (!ctx) return UGACHE_EINVAL;
+  if (dev_ptr) *dev_ptr = ctx->slab;
+  if (bytes) *bytes = ctx->slab_bytes;
+  if (n_slots) *n_slots = ctx->n_slots;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_ipc_handle(ugache_ctx *ctx, void *buf, size_t *len) {
+  if (!ctx || !buf || !len) return UGACHE_EINVAL;
+  if (*len < sizeof(cudaIpcMemHandle_t)) return UGACHE_EINVAL;
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  cudaIpcMemHandle_t h;
+  UG_CUDA(ctx, cudaIpcGetMemHandle(&h, ctx->slab));
+  memcpy(buf, &h, sizeof(h));
+  *len = sizeof(h);
+  return UGACHE_OK;
+}
+
+ugache_status ugache_open_peers(ugache_ctx *ctx, const void *all_handles, size_t len_each) {
+  if (!ctx || !all_handles || len_each < sizeof(cudaIpcMemHandle_t)) return UGACHE_EINVAL;
+  if (ctx->peers_ready && ctx->cfg.num_gpus > 1) return fail(ctx, UGACHE_ESTATE, "peers already set");
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  const uint8_t *hb = static_cast<const uint8_t *>(all_handles);
+  for (int j = 0; j < ctx->cfg.num_gpus; ++j) {
+    if (j == ctx->cfg.rank) continue;
+    cudaIpcMemHandle_t h;
+    memcpy(&h, hb + (size_t)j * len_each, sizeof(h));
+    void *p = nullptr;
+    cudaError_t e = cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) {
+      cuda_fail(ctx, e, "cudaIpcOpenMemHandle");
+      return UGACHE_EPEER;
+    }
+    ctx->ipc_mapped[j] = p;
+    ctx->src_base[j] = static_cast<const uint8_t *>(p);
+  }
+  ctx->peers_ready = true;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_set_peer_slabs(ugache_ctx *ctx, const void *const *slabs) {
+  if (!ctx || !slabs) return UGACHE_EINVAL;
+  for (int j = 0; j < ctx->cfg.num_gpus; ++j) {
+    if (j == ctx->cfg.rank) continue;
+    if (!slabs[j]) return UGACHE_EINVAL;
+    int dev = -1;
+    if (!is_device_pointer(slabs[j], &dev)) return fail(ctx, UGACHE_EPEER, "peer slab is not device memory");
+    if (dev != ctx->device) {
+      int can = 0;
+      cudaDeviceCanAccessPeer(&can, ctx->device, dev);
+      if (!can) return fail(ctx, UGACHE_EPEER, "no peer access to the slab's device");
+      ugache_status st = begin(ctx);
+      if (st != UGACHE_OK) return st;
+      cudaError_t e = cudaDeviceEnablePeerAccess(dev, 0);
+      if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) {
+        cuda_fail(ctx, e, "cudaDeviceEnablePeerAccess");
+        return UGACHE_EPEER;
+      }
+      (void)cudaGetLastError();
+    }
+    ctx->src_base[j] = static_cast<const uint8_t *>(slabs[j]);
+  }
+  ctx->peers_ready = true;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_fill(ugache_ctx *ctx, void *stream) {
+  if (!ctx) return UGACHE_EINVAL;
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (ctx->n_slots) {
+    ugk::FillParams fp;
+    fp.slot_keys = ctx->d_slot_keys;
+    fp.table = ctx->host_table_dev;
+    fp.slab = ctx->slab;
+    fp.n_slots = ctx->n_slots;
+    fp.row_bytes = ctx->cfg.row_bytes;
+    const int grid = ctx->sm_count * 8;
+    ugk::fill_kernel<<<grid, 256, 0, s>>>(fp);
+    UG_CUDA(ctx, cudaGetLastError());
+  }
+  ctx->filled = true;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_set_dedication(ugache_ctx *ctx, int32_t host_sms, int32_t peer_sms) {
+  if (!ctx || host_sms < 0 || peer_sms < 0) return UGACHE_EINVAL;
+  const int hs = host_sms ? host_sms : ctx->host_sms;
+  const int ps = peer_sms ? peer_sms : ctx->peer_sms;
+  const int G = ctx->cfg.num_gpus;
+  if (hs < 1 || hs > ctx->sm_count) return UGACHE_EINVAL;
+  if (G > 1 && (ps < 1 || (int64_t)hs + (int64_t)(G - 1) * ps > ctx->sm_count)) return UGACHE_EINVAL;
+  ctx->host_sms = hs;
+  ctx->peer_sms = ps;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_set_mode(ugache_ctx *ctx, int32_t mode) {
+  if (!ctx || (mode != UGACHE_MODE_FACTORED && mode != UGACHE_MODE_RANDOM_DISPATCH))
+    return UGACHE_EINVAL;
+  ctx->mode = mode;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type, uint64_t n,
+                             void *out, void *stream) {
+  if (!ctx) return UGACHE_EINVAL;
+  if (key_type != UGACHE_KEY_I64 && key_type != UGACHE_KEY_U32) return UGACHE_EINVAL;
+  if (n >= (1ull << 32)) return UGACHE_EINVAL;
+  if (!ctx->filled || !ctx->peers_ready) return fail(ctx, UGACHE_ESTATE, "extract before fill/peers");
+  ctx->last_n = n;
+  ctx->last_launches = 0;
+  ctx->timing_valid = false;
+  if (n == 0) return UGACHE_OK;
+  if (!keys || !out) return UGACHE_EINVAL;
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const uint32_t R = ctx->cfg.row_bytes;
+  const size_t key_bytes = key_type == UGACHE_KEY_I64 ? 8 : 4;
+
+  const void *dkeys = keys;
+  if (!is_device_pointer(keys, nullptr)) {
+    st = ensure_stage(ctx, &ctx->d_keys_stage, &ctx->keys_stage_bytes, n * key_bytes);
+    if (st != UGACHE_OK) return st;
+    UG_CUDA(ctx, cudaMemcpyAsync(ctx->d_keys_stage, keys, n * key_bytes, cudaMemcpyHostToDevice, s));
+    dkeys = ctx->d_keys_stage;
+  }
+  uint8_t *dout = static_cast<uint8_t *>(out);
+  const bool host_out = !is_device_pointer(out, nullptr);
+  if (host_out) {
+    st = ensure_stage(ctx, &ctx->d_out_stage, &ctx->out_stage_bytes, n * (size_t)R);
+    if (st != UGACHE_OK) return st;
+    dout = static_cast<uint8_t *>(ctx->d_out_stage);
+  } else if (reinterpret_cast<uintptr_t>(out) % 16 != 0) {
+    return fail(ctx, UGACHE_EINVAL, "out must be 16-byte aligned");
+  }
+
+  if (ctx->mode == UGACHE_MODE_RANDOM_DISPATCH) {
+    ugk::RandomParams rp;
+    rp.keys = dkeys;
+    rp.loc = ctx->d_loc;
+    rp.ctrl = ctx->d_ctrl;
+    for (int j = 0; j < ugk::kMaxSrc; ++j) rp.base[j] = ctx->src_base[j];
+    rp.out = dout;
+    rp.num_rows = ctx->cfg.num_rows;
+    rp.n = (uint32_t)n;
+    rp.row_bytes = R;
+    rp.num_src = ctx->cfg.num_gpus + 1;
+    if (ctx->timing) UG_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
+    if (ctx->timing) UG_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
+    if (key_type == UGACHE_KEY_I64)
+      ugk::random_dispatch_kernel<int64_t><<<ctx->sm_count, ugk::kGatherThreads, kOneCtaPerSmSmem, s>>>(rp);
+    else
+      ugk::random_dispatch_kernel<uint32_t><<<ctx->sm_count, ugk::kGatherThreads, kOneCtaPerSmSmem, s>>>(rp);
+    UG_CUDA(ctx, cudaGetLastError());
+    ctx->last_launches = 1;
+  } else {
+    st = ensure_scratch(ctx, n);
+    if (st != UGACHE_OK) return st;
+    ugk::LocateParams lp;
+    lp.keys = dkeys;
+    lp.loc = ctx->d_loc;
+    lp.buckets = ctx->d_buckets;
+    lp.ctrl = ctx->d_ctrl;
+    lp.out = dout;
+    lp.num_rows = ctx->cfg.num_rows;
+    lp.bucket_cap = ctx->bucket_cap;
+    lp.n = (uint32_t)n;
+    lp.row_bytes = R;
+    lp.num_src = ctx->cfg.num_gpus + 1;
+    const unsigned lgrid = (unsigned)((n + ugk::kLocateTile - 1) / ugk::kLocateTile);
+    if (ctx->timing) UG_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
+    if (key_type == UGACHE_KEY_I64)
+      ugk::locate_bucket_kernel<int64_t><<<lgrid, ugk::kLocateThreads, 0, s>>>(lp);
+    else
+      ugk::locate_bucket_kernel<uint32_t><<<lgrid, ugk::kLocateThreads, 0, s>>>(lp);
+    UG_CUDA(ctx, cudaGetLastError());
+    if (ctx->timing) UG_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
+
+    ugk::GatherParams gp;
+    gp.buckets = ctx->d_buckets;
+    gp.ctrl = ctx->d_ctrl;
+    for (int j = 0; j < ugk::kMaxSrc; ++j) gp.base[j] = ctx->src_base[j];
+    gp.out = dout;
+    gp.bucket_cap = ctx->bucket_cap;
+    gp.row_bytes = R;
+    gp.num_src = ctx->cfg.num_gpus + 1;
+    gp.local_src = ctx->cfg.rank;
+    int grid = 0;
+    build_roles(ctx, &gp, &grid);
+    ugk::factored_gather_kernel<<<grid, ugk::kGatherThreads, kOneCtaPerSmSmem, s>>>(gp);
+    UG_CUDA(ctx, cudaGetLastError());
+    ctx->last_launches = 2;
+  }
+  if (ctx->timing) {
+    UG_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));
+    ctx->timing_valid = true;
+  }
+  if (host_out) UG_CUDA(ctx, cudaMemcpyAsync(out, dout, n * (size_t)R, cudaMemcpyDeviceToHost, s));
+  ctx->last_stream = s;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_last_batch_stats(ugache_ctx *ctx, uint64_t *per_source, uint64_t *bad_keys) {
+  if (!ctx) return UGACHE_EINVAL;
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  const int S = ctx->cfg.num_gpus + 1;
+  if (ctx->last_n == 0 || ctx->last_launches == 0) {
+    if (per_source) for (int j = 0; j < S; ++j) per_source[j] = 0;
+    if (bad_keys) *bad_keys = 0;
+    return UGACHE_OK;
+  }
+  UG_CUDA(ctx, cudaStreamSynchronize(ctx->last_stream));
+  ugk::Ctrl c;
+  UG_CUDA(ctx, cudaMemcpy(&c, ctx->d_ctrl, sizeof(c), cudaMemcpyDeviceToHost));
+  if (per_source) for (int j = 0; j < S; ++j) per_source[j] = c.stat_counts[j];
+  if (bad_keys) *bad_keys = c.stat_bad;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_enable_timing(ugache_ctx *ctx, int32_t on) {
+  if (!ctx) return UGACHE_EINVAL;
+  ctx->timing = on != 0;
+  ctx->timing_valid = false;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_last_batch_timing(ugache_ctx *ctx, float *ms_locate, float *ms_gather) {
+  if (!ctx) return UGACHE_EINVAL;
+  if (!ctx->timing_valid) return fail(ctx, UGACHE_ESTATE, "no timed extract");
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  UG_CUDA(ctx, cudaEventSynchronize(ctx->ev[2]));
+  float a = 0, b = 0;
+  UG_CUDA(ctx, cudaEventElapsedTime(&a, ctx->ev[0], ctx->ev[1]));
+  UG_CUDA(ctx, cudaEventElapsedTime(&b, ctx->ev[1], ctx->ev[2]));
+  if (ms_locate) *ms_locate = a;
+  if (ms_gather) *ms_gather = b;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_last_launch_count(const ugache_ctx *ctx, int32_t *launches) {
+  if (!ctx || !launches) return UGACHE_EINVAL;
+  *launches = ctx->last_launches;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_export_placement(ugache_ctx *ctx, uint64_t *loc, uint64_t *slot_keys,
+                                      uint64_t *n_slots) {
+  if (!ctx) return UGACHE_EINVAL;
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  if (loc)
+    UG_CUDA(ctx, cudaMemcpy(loc, ctx->d_loc, ctx->cfg.num_rows * sizeof(uint64_t), cudaMemcpyDeviceToHost));
+  if (slot_keys && ctx->n_slots)
+    UG_CUDA(ctx, cudaMemcpy(slot_keys, ctx->d_slot_keys, ctx->n_slots * sizeof(uint64_t),
+                            cudaMemcpyDeviceToHost));
+  if (n_slots) *n_slots = ctx->n_slots;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_read_slab(ugache_ctx *ctx, uint64_t first, uint64_t count, void *dst) {
+  if (!ctx || (!dst && count)) return UGACHE_EINVAL;
+  if (first > ctx->plan.capacity_rows || count > ctx->plan.capacity_rows - first) return UGACHE_EINVAL;
+  if (!count) return UGACHE_OK;
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  const uint64_t R = ctx->cfg.row_bytes;
+  UG_CUDA(ctx, cudaDeviceSynchronize());
+  UG_CUDA(ctx, cudaMemcpy(dst, ctx->slab + first * R, count * R, cudaMemcpyDeviceToHost));
+  return UGACHE_OK;
+}
+
+ugache_status ugache_destroy(ugache_ctx *ctx) {
+  if (!ctx) return UGACHE_OK;
+  if (cudaSetDevice(ctx->device) == cudaSuccess) {
+    cudaDeviceSynchronize();
+    for (int j = 0; j < UGACHE_MAX_GPUS; ++j)
+      if (ctx->ipc_mapped[j]) cudaIpcCloseMemHandle(ctx->ipc_mapped[j]);
+    cudaFree(ctx->slab);
+    cudaFree(ctx->d_loc);
+    cudaFree(ctx->d_slot_keys);
+    cudaFree(ctx->d_ctrl);
+    cudaFree(ctx->d_buckets);
+    cudaFree(ctx->d_keys_stage);
+    cudaFree(ctx->d_out_stage);
+    for (int i = 0; i < 3; ++i)
+      if (ctx->ev[i]) cudaEventDestroy(ctx->ev[i]);
+  }
+  unregister_host_table(ctx);
+  (void)cudaGetLastError();
+  delete ctx;
+  return UGACHE_OK;
+}
+
+}  // extern "C"
