@@ -1,0 +1,440 @@
+#!/usr/bin/env python3
+"""bench.py -- UGache factored embedding extraction on B200 (one process per GPU).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload gnn_pa] [--cache-ratio 0.1]
+                  [--policy ugache|replication|partition] [--mode factored|random]
+                  [--impl ours|reference]
+
+A step is one ugache_extract of one batch (locate + bucket + factored gather, SURVEY.md
+8(a) rows A1-A4) per GPU.  Default workload: BASELINE.json configs[1] (Papers100M-shaped,
+111M x 128 fp32 rows = 56.8 GB host table, 500K unique Zipf(1.2) keys per GPU per batch,
+10 % per-GPU cache).  Prints ONE JSON line on rank 0.
+
+Timing: W warm-up steps; then K steps, each bracketed by CUDA events on the extract stream
+with a 256 MiB L2-flush write between steps (outside the events); barrier + synchronize
+on both sides; per-rank time = sum of the K event intervals; value = bytes of all ranks /
+max over ranks.  e2e: the same metric through UGache.extract with pinned HOST key and
+output buffers (H2D + extract + D2H inside the events).  --impl reference times the CPU
+oracle (oracle/gather.c) on the same batches.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "extraction GB/s (n*R/t_batch, all GPUs), ms/batch, % of source-mix roofline"
+
+
+def log(*a):
+    print("[bench]", *a, file=sys.stderr, flush=True)
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--workload", default="gnn_pa")
+    ap.add_argument("--cache-ratio", type=float, default=None)
+    ap.add_argument("--policy", default="ugache")
+    ap.add_argument("--mode", default="factored", choices=["factored", "random"])
+    ap.add_argument("--host-sms", type=int, default=0)
+    ap.add_argument("--peer-sms", type=int, default=0)
+    ap.add_argument("--batches", type=int, default=4, help="distinct batches cycled per rank")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--no-verify", action="store_true")
+    ap.add_argument("--extra", action="store_true", help="also time the random-dispatch ablation")
+    return ap.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, ws, local
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, index: int):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={index}", f"--query-gpu={q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        self.f.flush()
+        rows = []
+        with open(self.f.name) as fh:
+            for line in fh:
+                parts = [x.strip() for x in line.split(",")]
+                if len(parts) >= 9:
+                    rows.append(parts)
+        os.unlink(self.f.name)
+        if not rows:
+            return None
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i] == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": reasons,
+                "samples": len(rows)}
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f)
+    except Exception:
+        return {}
+
+
+def pcie_h2d_peak(torch) -> float:
+    """Live PCIe reference: pinned-host -> device cudaMemcpy of 1 GiB, best of 5 (GB/s)."""
+    n = 1 << 30
+    h = torch.empty(n, dtype=torch.uint8).pin_memory()
+    d = torch.empty(n, dtype=torch.uint8, device="cuda")
+    best = 1e9
+    for _ in range(5):
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s.record()
+        d.copy_(h, non_blocking=True)
+        e.record()
+        torch.cuda.synchronize()
+        best = min(best, s.elapsed_time(e))
+    del h, d
+    return n / (best * 1e-3) / 1e9
+
+
+def setup_table(wl, rank, ws, torch_dist):
+    import synth
+    t0 = time.time()
+    if ws == 1:
+        table = synth.HostTable(wl.num_rows, wl.row_bytes)
+        table.fill()
+    else:
+        path = f"/dev/shm/ugache_bench_{wl.name}_{os.getpid() if False else 'shared'}"
+        if rank == 0:
+            table = synth.HostTable(wl.num_rows, wl.row_bytes, shm_path=path, create=True)
+            table.fill()
+        torch_dist.barrier()
+        if rank != 0:
+            table = synth.HostTable(wl.num_rows, wl.row_bytes, shm_path=path, create=False)
+    log(f"table {wl.num_rows} x {wl.row_bytes} B = {wl.table_bytes / 1e9:.1f} GB ready in "
+        f"{time.time() - t0:.1f}s")
+    return table
+
+
+def make_batches(wl, rank, nb):
+    import synth
+    t0 = time.time()
+    b = [synth.make_batch(wl, rank, i) for i in range(nb)]
+    log(f"{nb} batches of {len(b[0])} keys in {time.time() - t0:.1f}s")
+    return b
+
+
+def run_reference(args, wl):
+    """--impl reference: the CPU oracle (plain OpenMP gather) on the box's host cores."""
+    import oracle
+    rank, ws, _ = dist_env()
+    if rank != 0:
+        return
+    import synth
+    table = synth.HostTable(wl.num_rows, wl.row_bytes)
+    table.fill()
+    batches = make_batches(wl, 0, max(1, min(args.batches, args.steps)))
+    n = len(batches[0])
+    out = np.empty((n, wl.row_bytes), dtype=np.uint8)
+    for i in range(args.warmup):
+        oracle.gather(table.ptr, wl.num_rows, wl.row_bytes, batches[i % len(batches)], out)
+    times = []
+    for i in range(args.steps):
+        t = time.perf_counter()
+        oracle.gather(table.ptr, wl.num_rows, wl.row_bytes, batches[i % len(batches)], out)
+        times.append(time.perf_counter() - t)
+    tot = sum(times)
+    gbs = args.steps * n * wl.row_bytes / tot / 1e9
+    cores = len(os.sched_getaffinity(0))
+    line = {"metric": METRIC, "value": gbs, "unit": "GB/s", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": tot / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
+            "data": "synthetic", "impl": "reference",
+            "config": config_dict(args, wl, ws),
+            "cpu_baseline": {"value": gbs, "unit": "GB/s", "cores": cores, "kind": "oracle",
+                             "sample": f"{args.steps} full batches of {n} keys (oracle/gather.c, "
+                                       f"OpenMP, {cores} threads) on rank 0"},
+            "e2e": {"value": gbs, "unit": "GB/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def config_dict(args, wl, ws):
+    return {"workload": wl.name, "num_rows": wl.num_rows, "row_bytes": wl.row_bytes,
+            "payload": f"{wl.row_bytes // (2 if wl.dtype == 'f16' else 4)} x {wl.dtype}",
+            "keys_per_batch_per_gpu": wl.keys_per_batch, "batch_kind": wl.batch_kind,
+            "alpha": wl.alpha, "cache_ratio": args.cache_ratio if args.cache_ratio is not None
+            else wl.cache_ratio, "policy": args.policy, "mode": args.mode,
+            "parallelism": f"dp{ws}",
+            "l2": "256 MiB L2-flush write between timed steps (outside the events); per-step "
+                  "output > L2"}
+
+
+def main():
+    args = parse()
+    import synth
+    wl = synth.get_workload(args.workload)
+    if args.cache_ratio is not None:
+        from dataclasses import replace
+        wl = replace(wl, cache_ratio=args.cache_ratio)
+    if args.impl == "reference":
+        run_reference(args, wl)
+        return
+
+    import torch
+    import torch.distributed as tdist
+    import oracle
+    from paper_conf_sosp_songz0c23_b200 import UGache, dist as ugdist, make_config, solve
+    rank, ws, local = dist_env()
+    if ws != args.gpus:
+        log(f"warning: --gpus {args.gpus} but WORLD_SIZE {ws}; using WORLD_SIZE")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if ws > 1:
+        tdist.init_process_group("nccl", device_id=dev)
+
+    table = setup_table(wl, rank, ws, tdist)
+    t0 = time.time()
+    h = synth.hotness(wl)
+    log(f"hotness in {time.time() - t0:.1f}s")
+    C = wl.capacity_rows
+    cfg = make_config(wl.num_rows, wl.row_bytes, C, num_gpus=ws, rank=rank, device=local,
+                      policy=args.policy, host_sms=args.host_sms, peer_sms=args.peer_sms)
+    t0 = time.time()
+    plan, order = solve(cfg, h)
+    log(f"solve in {time.time() - t0:.1f}s: k={plan.k} band_end={plan.band_end} z={plan.z:.3e}")
+    del h
+    t0 = time.time()
+    cache = UGache(table, wl.num_rows, wl.row_bytes, C, num_gpus=ws, rank=rank, device=local,
+                   policy=args.policy, plan=plan, order=order, host_sms=args.host_sms,
+                   peer_sms=args.peer_sms)
+    log(f"init (register host table, location table, slab) in {time.time() - t0:.1f}s")
+    ugdist.connect(cache, order=order)
+    del order
+    stream = torch.cuda.Stream(device=dev)
+    t0 = time.time()
+    cache.fill(stream)
+    stream.synchronize()
+    ugdist.barrier()
+    log(f"fill in {time.time() - t0:.2f}s")
+    if args.mode == "random":
+        cache.set_mode("random")
+
+    batches = make_batches(wl, rank, max(1, min(args.batches, args.steps + args.warmup)))
+    n = len(batches[0])
+    R = wl.row_bytes
+    dkeys = [torch.from_numpy(b).to(dev) for b in batches]
+    out = torch.empty((n, R), dtype=torch.uint8, device=dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    cache.enable_timing(True)
+
+    def step(i, timed):
+        with torch.cuda.stream(stream):
+            flush.fill_(i & 0xFF)  # evict L2 between steps (outside the events)
+        if timed:
+            s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            s.record(stream)
+        cache.extract(dkeys[i % len(dkeys)], out, stream)
+        if timed:
+            e.record(stream)
+            return s, e
+        return None
+
+    for i in range(args.warmup):
+        step(i, False)
+    stream.synchronize()
+    ugdist.barrier()
+    torch.cuda.synchronize()
+    clocks = Clocks(local) if rank == 0 else None
+    time.sleep(0.3 if clocks else 0)
+    evs, loc_ms, gat_ms, per_src = [], [], [], []
+    launches = 0
+    for i in range(args.steps):
+        evs.append(step(args.warmup + i, True))
+        a, b = cache.last_batch_timing()   # syncs this step's gather (after its end event)
+        loc_ms.append(a)
+        gat_ms.append(b)
+        per, _ = cache.last_batch_stats()
+        per_src.append(per)
+        launches += cache.last_launch_count()
+    stream.synchronize()
+    torch.cuda.synchronize()
+    ugdist.barrier()
+    clk = clocks.stop() if clocks else None
+    step_ms = [s.elapsed_time(e) for s, e in evs]
+    my_total_s = sum(step_ms) / 1e3
+    max_total_s = ugdist.max_over_ranks(my_total_s)
+    bytes_all = ugdist.sum_over_ranks(float(args.steps * n * R))
+    value = bytes_all / max_total_s / 1e9
+
+    # ---- parity on the full-size batch (every key, byte for byte) -------------------
+    parity = None
+    if not args.no_verify:
+        cache.extract(dkeys[0], out, stream)
+        stream.synchronize()
+        ref, _ = oracle.gather(table.ptr, wl.num_rows, R, batches[0])
+        parity = "bit-exact" if np.array_equal(out.cpu().numpy(), ref) else "MISMATCH"
+        del ref
+
+    # ---- e2e through the public API with pinned host buffers -------------------------
+    hkeys = [torch.from_numpy(b).pin_memory() for b in batches]
+    hout = torch.empty((n, R), dtype=torch.uint8).pin_memory()
+    cache.enable_timing(False)
+    cache.extract(hkeys[0], hout, stream)  # warm the staging buffers
+    stream.synchronize()
+    e2e_ms = []
+    for i in range(args.e2e_steps):
+        with torch.cuda.stream(stream):
+            flush.fill_(i & 0xFF)
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s.record(stream)
+        cache.extract(hkeys[i % len(hkeys)], hout, stream)
+        e.record(stream)
+        stream.synchronize()
+        e2e_ms.append(s.elapsed_time(e))
+    e2e_total = ugdist.max_over_ranks(sum(e2e_ms) / 1e3)
+    e2e_bytes = ugdist.sum_over_ranks(float(args.e2e_steps * n * R))
+    e2e_value = e2e_bytes / e2e_total / 1e9
+
+    # ---- optional FEM ablation: random dispatch through the same locate table -------
+    ablation = None
+    if args.extra and args.mode == "factored":
+        cache.set_mode("random")
+        cache.enable_timing(True)
+        rms = []
+        for i in range(args.steps + 2):
+            r = step(i, True)
+            if i >= 2:
+                stream.synchronize()
+                rms.append(r[0].elapsed_time(r[1]))
+        cache.set_mode("factored")
+        ablation = {"random_dispatch_ms_per_step": statistics.mean(rms),
+                    "factored_ms_per_step": statistics.mean(step_ms)}
+
+    # ---- roofline --------------------------------------------------------------------
+    peaks = measured_peaks()
+    hbm = float(peaks.get("hbm_gbs", 6650.0))
+    hbm_src = "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "B200_PROFILING.md fallback"
+    pcie = pcie_h2d_peak(torch) if rank == 0 else 0.0
+    per = np.mean(np.stack(per_src), axis=0)
+    G = ws
+    n_local = float(per[rank]) if G > 0 else 0.0
+    n_host = float(per[G])
+    n_peer = float(per.sum() - n_local - n_host)
+    kb = 8
+    gat_s = statistics.mean(gat_ms) / 1e3
+    loc_s = statistics.mean(loc_ms) / 1e3
+    # algorithmic bytes of the gather kernel: rows read per source + rows written + bucket reads
+    gather_hbm_bytes = n_local * R + n * R + n * 8
+    gather_pcie_bytes = n_host * R
+    t_hbm = gather_hbm_bytes / (hbm * 1e9)
+    t_pcie = gather_pcie_bytes / (pcie * 1e9) if pcie else 0.0
+    nvl = 770.0
+    t_nvl = n_peer * R / (nvl * 1e9)
+    terms = {"hbm": t_hbm, "pcie": t_pcie, "nvlink": t_nvl}
+    bound = max(terms, key=terms.get)
+    if bound == "hbm":
+        achieved, peak, unit, psrc = gather_hbm_bytes / gat_s / 1e9, hbm, "GB/s", hbm_src
+    elif bound == "pcie":
+        achieved, peak, unit, psrc = gather_pcie_bytes / gat_s / 1e9, pcie, "GB/s", \
+            "live cudaMemcpy pinned H2D 1 GiB best-of-5 in this run"
+    else:
+        achieved, peak, unit, psrc = n_peer * R / gat_s / 1e9, nvl, "GB/s", \
+            "B200_PROFILING.md measured peer copy"
+    # whole-step source-mix roofline (locate + gather): every byte the step moves
+    step_hbm = (n * kb + n * 32 + n * 8 + n * 8) + gather_hbm_bytes
+    t_roof = max(step_hbm / (hbm * 1e9), t_pcie, t_nvl)
+    ms_per_step = statistics.mean(step_ms)
+    line = {
+        "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": ws, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": config_dict(args, wl, ws),
+        "roofline": {"bound": bound, "achieved": achieved, "peak": peak, "unit": unit,
+                     "frac": achieved / peak if peak else None, "traffic": None,
+                     "kernel": "factored_gather_kernel", "peak_source": psrc,
+                     "kernel_ms": statistics.mean(gat_ms)},
+        "source_mix_roofline": {"t_roof_us": t_roof * 1e6, "t_step_us": ms_per_step * 1e3,
+                                "frac": t_roof / (ms_per_step / 1e3),
+                                "terms_us": {"hbm": step_hbm / (hbm * 1e9) * 1e6,
+                                             "pcie": t_pcie * 1e6, "nvlink": t_nvl * 1e6},
+                                "bw_gbs": {"hbm": hbm, "pcie": pcie, "nvlink": nvl}},
+        "per_source_keys": {"local": n_local, "peer": n_peer, "host": n_host},
+        "kernel_ms": {"locate_bucket": statistics.mean(loc_ms), "factored_gather": statistics.mean(gat_ms)},
+        "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": n * 8,
+                "d2h_bytes_per_step": n * R, "ms_per_step": statistics.mean(e2e_ms)},
+        "gpu_launches": launches,
+        "clocks": clk,
+        "parity": parity,
+        "plan": {"k": plan.k, "band_end": plan.band_end, "capacity_rows": plan.capacity_rows,
+                 "host_sms": plan.host_sms, "peer_sms": plan.peer_sms,
+                 "z_model_us": plan.z * 1e6, "z_replication_us": plan.z_replication * 1e6,
+                 "z_partition_us": plan.z_partition * 1e6},
+    }
+    if ablation:
+        line["fem_ablation"] = ablation
+
+    # ---- CPU oracle baseline (rank 0, N=1 only, bounded sample, after GPU timing) ----
+    if rank == 0 and ws == 1:
+        out_np = np.empty((n, R), dtype=np.uint8)
+        t_end = time.perf_counter() + args.cpu_seconds
+        done, cpu_t = 0, 0.0
+        while time.perf_counter() < t_end or done == 0:
+            b = batches[done % len(batches)]
+            t = time.perf_counter()
+            oracle.gather(table.ptr, wl.num_rows, R, b, out_np)
+            cpu_t += time.perf_counter() - t
+            done += 1
+        cores = len(os.sched_getaffinity(0))
+        line["cpu_baseline"] = {"value": done * n * R / cpu_t / 1e9, "unit": "GB/s",
+                                "cores": cores, "kind": "oracle",
+                                "sample": f"{done} batches x {n} keys of {wl.name} "
+                                          f"(~{args.cpu_seconds:.0f}s, OpenMP {cores} threads)",
+                                "ms_per_batch": cpu_t / done * 1e3}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    cache.close()
+    table.close()
+    if ws > 1:
+        tdist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -176,6 +176,12 @@ ugache_status ugache_set_dedication(ugache_ctx *ctx, int32_t host_sms, int32_t p
 /* ugache_mode; FACTORED by default. */
 ugache_status ugache_set_mode(ugache_ctx *ctx, int32_t mode);
 
+/* Host-source read order (B200 box property): when on (default),
+ * the host CTAs of the factored gather first order the host bucket by key range so the
+ * rows in flight cover a small window of host address space, then copy in that order.
+ * off = copy in bucket order.  Output is identical either way. */
+ugache_status ugache_set_host_ordering(ugache_ctx *ctx, int32_t on);
+
 /* Per-source key counts of the last extract: per_source[j] for GPU j (j == rank: local),
  * per_source[G] for host (G+1 entries); bad_keys: out-of-range keys.  Synchronises with
  * the last extract.  Per-source hit rates as in Fig. 14. */

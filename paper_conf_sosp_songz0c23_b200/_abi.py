@@ -73,6 +73,7 @@ SIGNATURES = {
     "ugache_extract": (_ST, [_P, _P, _c.c_int32, _c.c_uint64, _P, _P]),
     "ugache_set_dedication": (_ST, [_P, _c.c_int32, _c.c_int32]),
     "ugache_set_mode": (_ST, [_P, _c.c_int32]),
+    "ugache_set_host_ordering": (_ST, [_P, _c.c_int32]),
     "ugache_last_batch_stats": (_ST, [_P, _P, ctypes.POINTER(_c.c_uint64)]),
     "ugache_enable_timing": (_ST, [_P, _c.c_int32]),
     "ugache_last_batch_timing": (_ST, [_P, ctypes.POINTER(_c.c_float), ctypes.POINTER(_c.c_float)]),

@@ -29,6 +29,7 @@ constexpr int kGatherWarps = kGatherThreads / 32;
 constexpr int kRowsInFlight = 8;     // rows per warp per step (U)
 constexpr int kLocalChunk = 64;      // rows per local-cursor claim
 constexpr uint32_t kFullMask = 0xFFFFFFFFu;
+constexpr int kMaxSmId = 256;        // role table size, indexed by %smid
 
 // Device control block (one per ctx).  counts/local_cursor/done/bad are consumed and reset
 // by the last CTA of every gather launch, so consecutive extracts need no memset.
@@ -39,8 +40,16 @@ struct Ctrl {
   uint32_t bad;
   uint32_t stat_counts[kMaxSrc];
   uint32_t stat_bad;
-  uint32_t pad[4];
+  uint32_t host_arrive[2];  // intra-role barriers of the host CTAs
+  uint32_t host_cursor;     // dynamic cursor over the range-ordered host bucket
+  uint32_t pad;
 };
+
+// Host-bucket range ordering: host rows are read in ascending
+// key-range order so that the rows in flight span a small window of host address space
+// (IOMMU/ATS translation reach), instead of the whole table.
+constexpr int kMaxRanges = 4096;
+constexpr uint32_t kHostSortMin = 4096;  // below this many host keys, read unordered
 
 struct LocateParams {
   const void *keys;
@@ -66,7 +75,16 @@ struct GatherParams {
   int32_t local_src;
   int32_t n_roles;
   int32_t role_src[kMaxSrc];       // role r serves source role_src[r]
-  int32_t role_cta_end[kMaxSrc];   // CTAs [role_cta_end[r-1], role_cta_end[r]) have role r
+  int32_t role_count[kMaxSrc];     // number of SMs (= CTAs) with role r
+  uint8_t sm_role[kMaxSmId];       // role of the CTA running on SM %smid
+  uint8_t sm_role_idx[kMaxSmId];   // its index within the role
+  // host range ordering
+  uint64_t *host_sorted;           // bucket_cap entries of scratch
+  uint32_t *range_count;           // kMaxRanges, zero between launches
+  uint32_t *range_cursor;          // kMaxRanges, zero between launches
+  uint32_t range_shift;            // range = row >> range_shift
+  uint32_t n_ranges;               // <= kMaxRanges
+  int32_t host_sort;               // 0 = read the host bucket in bucket order
 };
 
 struct RandomParams {
@@ -165,6 +183,9 @@ __device__ __forceinline__ void finish_launch(Ctrl *ctrl, int num_src) {
       c->stat_bad = c->bad;
       c->bad = 0;
       c->local_cursor = 0;
+      c->host_arrive[0] = 0;
+      c->host_arrive[1] = 0;
+      c->host_cursor = 0;
       __threadfence();
       c->done = 0;
     }
@@ -235,24 +256,125 @@ __global__ void __launch_bounds__(kLocateThreads)
   }
 }
 
+// Barrier among the `n` CTAs of one role.  The gather kernel is launched cooperatively
+// (one CTA per SM), so every CTA of a role is co-resident.
+__device__ __forceinline__ void role_barrier(uint32_t *ctr, uint32_t n) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    atomicAdd(ctr, 1u);
+    uint32_t v;
+    do {
+      asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+      if (v < n) __nanosleep(64);
+    } while (v < n);
+  }
+  __syncthreads();
+}
+
+// Exclusive scan of src[0..n) (global) into dst[0..n) (shared); n <= kMaxRanges.
+__device__ __forceinline__ void block_exclusive_scan(const uint32_t *src, uint32_t *dst, uint32_t n) {
+  __shared__ uint32_t s_warp[32];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nt = blockDim.x;
+  const uint32_t per = (n + nt - 1) / nt;
+  const uint32_t lo = min(n, tid * per), hi = min(n, lo + per);
+  uint32_t sum = 0;
+  for (uint32_t i = lo; i < hi; ++i) sum += src[i];
+  uint32_t incl = sum;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(kFullMask, incl, o);
+    if (lane >= o) incl += y;
+  }
+  if (lane == 31) s_warp[warp] = incl;
+  __syncthreads();
+  if (warp == 0) {
+    const int nw = nt >> 5;
+    uint32_t w = lane < nw ? s_warp[lane] : 0, wi = w;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(kFullMask, wi, o);
+      if (lane >= o) wi += y;
+    }
+    if (lane < nw) s_warp[lane] = wi - w;
+  }
+  __syncthreads();
+  uint32_t run = s_warp[warp] + incl - sum;
+  for (uint32_t i = lo; i < hi; ++i) {
+    const uint32_t v = src[i];
+    dst[i] = run;
+    run += v;
+  }
+  __syncthreads();
+}
+
+// Host role with range ordering: histogram -> barrier -> scan -> scatter -> barrier ->
+// dynamic in-order copy.  All host CTAs cooperate; `h`/`H` = index/count within the role.
+__device__ __forceinline__ void host_role_sorted(const GatherParams &p, const uint64_t *b,
+                                                 uint32_t cnt, int h, int H, uint32_t *s_tab) {
+  const int tid = threadIdx.x, lane = tid & 31;
+  const uint32_t lo = (uint32_t)((uint64_t)cnt * h / H), hi = (uint32_t)((uint64_t)cnt * (h + 1) / H);
+  for (uint32_t i = tid; i < p.n_ranges; i += blockDim.x) s_tab[i] = 0;
+  __syncthreads();
+  for (uint32_t e = lo + tid; e < hi; e += blockDim.x)
+    atomicAdd(&s_tab[(uint32_t)(b[e] >> 32) >> p.range_shift], 1u);
+  __syncthreads();
+  for (uint32_t i = tid; i < p.n_ranges; i += blockDim.x)
+    if (s_tab[i]) atomicAdd(&p.range_count[i], s_tab[i]);
+  role_barrier(&p.ctrl->host_arrive[0], (uint32_t)H);
+  block_exclusive_scan(p.range_count, s_tab, p.n_ranges);
+  for (uint32_t e = lo + tid; e < hi; e += blockDim.x) {
+    const uint64_t ent = b[e];
+    const uint32_t r = (uint32_t)(ent >> 32) >> p.range_shift;
+    p.host_sorted[s_tab[r] + atomicAdd(&p.range_cursor[r], 1u)] = ent;
+  }
+  role_barrier(&p.ctrl->host_arrive[1], (uint32_t)H);
+  {  // every host CTA is past its scatter: re-arm my slice of the range counters
+    const uint32_t zlo = p.n_ranges * h / H, zhi = p.n_ranges * (h + 1) / H;
+    for (uint32_t i = zlo + tid; i < zhi; i += blockDim.x) {
+      p.range_count[i] = 0;
+      p.range_cursor[i] = 0;
+    }
+  }
+  const uint8_t *base = p.base[p.num_src - 1];
+  uint32_t next = 0;
+  if (lane == 0) next = atomicAdd(&p.ctrl->host_cursor, (uint32_t)kRowsInFlight);
+  next = __shfl_sync(kFullMask, next, 0);
+  while (next < cnt) {
+    const uint32_t e0 = next;
+    if (lane == 0) next = atomicAdd(&p.ctrl->host_cursor, (uint32_t)kRowsInFlight);
+    next = __shfl_sync(kFullMask, next, 0);
+    copy_rows<kRowsInFlight>(base, p.out, p.row_bytes, p.host_sorted + e0,
+                             (int)min((uint32_t)kRowsInFlight, cnt - e0), lane);
+  }
+}
+
 // ---------------------------------------------------------------------------- K2
 __global__ void __launch_bounds__(kGatherThreads, 1)
     factored_gather_kernel(const GatherParams p) {
+  extern __shared__ __align__(16) uint32_t s_dyn[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  int r = 0;
-  while (r < p.n_roles - 1 && (int)blockIdx.x >= p.role_cta_end[r]) ++r;
+  // Role of this CTA = role of the SM it runs on (one CTA per SM, cooperative launch):
+  // the B200 replacement of the paper's MPS core limits.
+  uint32_t smid;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+  const int r = smid < (uint32_t)kMaxSmId ? p.sm_role[smid] : p.n_roles - 1;
   const int my_src = p.role_src[r];
-  const int cta_begin = r ? p.role_cta_end[r - 1] : 0;
-  const int role_ctas = p.role_cta_end[r] - cta_begin;
+  const int my_idx = smid < (uint32_t)kMaxSmId ? p.sm_role_idx[smid] : 0;
+  const int role_ctas = p.role_count[r];
   const uint32_t R = p.row_bytes;
 
-  if (my_src != p.local_src) {
+  const int host_src = p.num_src - 1;
+  if (my_src == host_src && p.host_sort && p.ctrl->counts[host_src] >= kHostSortMin) {
+    host_role_sorted(p, p.buckets + (uint64_t)host_src * p.bucket_cap, p.ctrl->counts[host_src],
+                     my_idx, role_ctas, s_dyn);
+  } else if (my_src != p.local_src) {
     // dedicated non-local extraction: static warp striding over this source's bucket
     const uint32_t cnt = p.ctrl->counts[my_src];
     const uint64_t *b = p.buckets + (uint64_t)my_src * p.bucket_cap;
     const uint8_t *base = p.base[my_src];
     const uint32_t W = (uint32_t)role_ctas * kGatherWarps;
-    const uint32_t gw = (uint32_t)((int)blockIdx.x - cta_begin) * kGatherWarps + warp;
+    const uint32_t gw = (uint32_t)my_idx * kGatherWarps + warp;
     for (uint32_t e0 = gw * kRowsInFlight; e0 < cnt; e0 += W * kRowsInFlight)
       copy_rows<kRowsInFlight>(base, p.out, R, b + e0, (int)min((uint32_t)kRowsInFlight, cnt - e0),
                                lane);
@@ -330,6 +452,16 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
   if (threadIdx.x < p.num_src && s_cnt[threadIdx.x])
     atomicAdd(&p.ctrl->counts[threadIdx.x], s_cnt[threadIdx.x]);
   finish_launch(p.ctrl, p.num_src);
+}
+
+// ---------------------------------------------------------------------------- probe
+// One CTA per SM (cooperative launch): record the %smid values of this device.
+__global__ void __launch_bounds__(32, 1) smid_probe_kernel(uint32_t *smids) {
+  if (threadIdx.x == 0) {
+    uint32_t smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    smids[blockIdx.x] = smid;
+  }
 }
 
 // ---------------------------------------------------------------------------- K5

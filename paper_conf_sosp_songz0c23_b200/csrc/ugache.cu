@@ -45,6 +45,11 @@ struct ugache_ctx {
   size_t keys_stage_bytes = 0;
   void *d_out_stage = nullptr;
   size_t out_stage_bytes = 0;
+  uint64_t *d_host_sorted = nullptr;
+  uint32_t *d_ranges = nullptr;  // 2 * kMaxRanges counters
+  uint32_t range_shift = 0, n_ranges = 1;
+  int host_sort = 1;
+  std::vector<int> smids;  // sorted %smid values of the device (one per SM)
   // dedication / mode
   int host_sms = 0, peer_sms = 0;
   int mode = UGACHE_MODE_FACTORED;
@@ -156,8 +161,13 @@ ugache_status ensure_scratch(ugache_ctx *ctx, uint64_t n) {
     ctx->d_buckets = nullptr;
     ctx->bucket_cap = 0;
   }
+  if (ctx->d_host_sorted) {
+    cudaFree(ctx->d_host_sorted);
+    ctx->d_host_sorted = nullptr;
+  }
   const size_t bytes = (size_t)(ctx->cfg.num_gpus + 1) * cap * sizeof(uint64_t);
   UG_CUDA(ctx, cudaMalloc(&ctx->d_buckets, bytes));
+  UG_CUDA(ctx, cudaMalloc(&ctx->d_host_sorted, cap * sizeof(uint64_t)));
   ctx->bucket_cap = cap;
   return UGACHE_OK;
 }
@@ -175,26 +185,44 @@ ugache_status ensure_stage(ugache_ctx *ctx, void **buf, size_t *have, size_t nee
   return UGACHE_OK;
 }
 
-// Role table of the gather kernel: host first, then each peer, then local.
+// Role table of the gather kernel: host SMs, then each peer's SMs, local
+// gets the rest.  SMs are handed out along a stride permutation of the sorted SM ids so
+// every role is spread over the whole chip (all GPCs / both dies) -- on the B200 box the
+// host source's zero-copy throughput scales with the number of GPCs issuing requests.
 void build_roles(const ugache_ctx *ctx, ugk::GatherParams *gp, int *grid) {
-  const int G = ctx->cfg.num_gpus, me = ctx->cfg.rank, S = ctx->sm_count;
-  int nr = 0, end = 0;
+  const int G = ctx->cfg.num_gpus, me = ctx->cfg.rank;
+  const int S = (int)ctx->smids.size();
+  int nr = 0;
+  std::vector<int> want;
   gp->role_src[nr] = G;  // host
-  end += ctx->host_sms;
-  gp->role_cta_end[nr++] = end;
+  want.push_back(ctx->host_sms);
+  ++nr;
   for (int j = 0; j < G; ++j) {
     if (j == me) continue;
-    gp->role_src[nr] = j;
-    end += ctx->peer_sms;
-    gp->role_cta_end[nr++] = end;
+    gp->role_src[nr++] = j;
+    want.push_back(ctx->peer_sms);
   }
-  if (end < S) {
-    gp->role_src[nr] = me;
-    end = S;
-    gp->role_cta_end[nr++] = end;
+  int used = 0;
+  for (int w : want) used += w;
+  if (used < S) {
+    gp->role_src[nr++] = me;
+    want.push_back(S - used);
   }
   gp->n_roles = nr;
-  *grid = end;
+  memset(gp->sm_role, nr - 1, sizeof(gp->sm_role));
+  memset(gp->sm_role_idx, 0, sizeof(gp->sm_role_idx));
+  int stride = (int)(S * 0.6180339887) | 1;
+  while (std::__gcd(stride, S) != 1) stride += 2;
+  int pos = 0;
+  for (int r = 0; r < nr; ++r) {
+    gp->role_count[r] = want[r];
+    for (int i = 0; i < want[r]; ++i, ++pos) {
+      const int sm = ctx->smids[(size_t)((int64_t)pos * stride % S)];
+      gp->sm_role[sm] = (uint8_t)r;
+      gp->sm_role_idx[sm] = (uint8_t)i;
+    }
+  }
+  *grid = S;
 }
 
 ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void *host_table,
@@ -229,12 +257,37 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   }
   UG_CUDA(ctx, cudaMalloc(&ctx->d_ctrl, sizeof(ugk::Ctrl)));
   UG_CUDA(ctx, cudaMemset(ctx->d_ctrl, 0, sizeof(ugk::Ctrl)));
+  UG_CUDA(ctx, cudaMalloc(&ctx->d_ranges, 2 * ugk::kMaxRanges * sizeof(uint32_t)));
+  UG_CUDA(ctx, cudaMemset(ctx->d_ranges, 0, 2 * ugk::kMaxRanges * sizeof(uint32_t)));
+  // host key ranges: the smallest power-of-two rows per range giving <= kMaxRanges ranges
+  ctx->range_shift = 0;
+  while (((N - 1) >> ctx->range_shift) + 1 > (uint64_t)ugk::kMaxRanges) ++ctx->range_shift;
+  ctx->n_ranges = (uint32_t)(((N - 1) >> ctx->range_shift) + 1);
   for (int i = 0; i < 3; ++i) UG_CUDA(ctx, cudaEventCreate(&ctx->ev[i]));
   ctx->src_base[cfg->rank] = ctx->slab;
   ctx->src_base[G] = ctx->host_table_dev;
   ctx->peers_ready = (G == 1);
   ctx->host_sms = ctx->plan.host_sms;
   ctx->peer_sms = ctx->plan.peer_sms;
+  {  // SM ids of this device (role table index)
+    uint32_t *d_ids = nullptr;
+    UG_CUDA(ctx, cudaMalloc(&d_ids, ctx->sm_count * sizeof(uint32_t)));
+    UG_CUDA(ctx, cudaFuncSetAttribute(ugk::smid_probe_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      (int)kOneCtaPerSmSmem));
+    void *args[] = {&d_ids};
+    cudaError_t e = cudaLaunchCooperativeKernel((const void *)ugk::smid_probe_kernel, dim3(ctx->sm_count),
+                                                dim3(32), args, kOneCtaPerSmSmem, nullptr);
+    std::vector<uint32_t> ids(ctx->sm_count);
+    if (e == cudaSuccess) e = cudaMemcpy(ids.data(), d_ids, ids.size() * 4, cudaMemcpyDeviceToHost);
+    cudaFree(d_ids);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "smid probe");
+    std::sort(ids.begin(), ids.end());
+    for (size_t i = 0; i < ids.size(); ++i) {
+      if (ids[i] >= (uint32_t)ugk::kMaxSmId || (i && ids[i] == ids[i - 1]))
+        return fail(ctx, UGACHE_ECUDA, "unexpected %smid layout");
+      ctx->smids.push_back((int)ids[i]);
+    }
+  }
   UG_CUDA(ctx, cudaFuncSetAttribute(ugk::factored_gather_kernel,
                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem));
   UG_CUDA(ctx, cudaFuncSetAttribute(ugk::random_dispatch_kernel<int64_t>,
@@ -450,6 +503,12 @@ ugache_status ugache_set_mode(ugache_ctx *ctx, int32_t mode) {
   return UGACHE_OK;
 }
 
+ugache_status ugache_set_host_ordering(ugache_ctx *ctx, int32_t on) {
+  if (!ctx) return UGACHE_EINVAL;
+  ctx->host_sort = on != 0;
+  return UGACHE_OK;
+}
+
 ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type, uint64_t n,
                              void *out, void *stream) {
   if (!ctx) return UGACHE_EINVAL;
@@ -535,10 +594,17 @@ ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type
     gp.row_bytes = R;
     gp.num_src = ctx->cfg.num_gpus + 1;
     gp.local_src = ctx->cfg.rank;
+    gp.host_sorted = ctx->d_host_sorted;
+    gp.range_count = ctx->d_ranges;
+    gp.range_cursor = ctx->d_ranges + ugk::kMaxRanges;
+    gp.range_shift = ctx->range_shift;
+    gp.n_ranges = ctx->n_ranges;
+    gp.host_sort = ctx->host_sort;
     int grid = 0;
     build_roles(ctx, &gp, &grid);
-    ugk::factored_gather_kernel<<<grid, ugk::kGatherThreads, kOneCtaPerSmSmem, s>>>(gp);
-    UG_CUDA(ctx, cudaGetLastError());
+    void *kargs[] = {&gp};
+    UG_CUDA(ctx, cudaLaunchCooperativeKernel((const void *)ugk::factored_gather_kernel, dim3(grid),
+                                             dim3(ugk::kGatherThreads), kargs, kOneCtaPerSmSmem, s));
     ctx->last_launches = 2;
   }
   if (ctx->timing) {
@@ -634,6 +700,8 @@ ugache_status ugache_destroy(ugache_ctx *ctx) {
     cudaFree(ctx->d_buckets);
     cudaFree(ctx->d_keys_stage);
     cudaFree(ctx->d_out_stage);
+    cudaFree(ctx->d_host_sorted);
+    cudaFree(ctx->d_ranges);
     for (int i = 0; i < 3; ++i)
       if (ctx->ev[i]) cudaEventDestroy(ctx->ev[i]);
   }

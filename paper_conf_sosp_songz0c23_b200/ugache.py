@@ -136,6 +136,9 @@ class UGache:
         m = {"factored": _abi.MODE_FACTORED, "random": _abi.MODE_RANDOM_DISPATCH}[mode]
         check(lib().ugache_set_mode(self.ctx, m), "ugache_set_mode", self.ctx)
 
+    def set_host_ordering(self, on: bool):
+        check(lib().ugache_set_host_ordering(self.ctx, int(on)), "ugache_set_host_ordering", self.ctx)
+
     def enable_timing(self, on: bool = True):
         check(lib().ugache_enable_timing(self.ctx, int(on)), "ugache_enable_timing", self.ctx)
 

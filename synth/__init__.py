@@ -262,25 +262,21 @@ def make_batch(wl: Workload, rank: int, batch_idx: int, return_draws: bool = Fal
 
 
 def expected_draws_unique(num: int, alpha: float, target: int) -> float:
-    """m such that sum_r 1-(1-p(r))^m = target (bisection in log-space)."""
-    p = zipf_pmf(num, alpha)
-    lp = np.log1p(-p)
-
-    def uniq(m):
-        return float(np.sum(-np.expm1(m * lp)))
-
-    lo, hi = float(target), float(target)
-    while uniq(hi) < target:
-        hi *= 2.0
-    for _ in range(50):
-        mid = math.sqrt(lo * hi)
-        if uniq(mid) < target:
-            lo = mid
-        else:
-            hi = mid
-        if hi / lo < 1 + 1e-7:
+    """m such that sum_r 1-(1-p(r))^m = target.  f(m) is increasing and concave, so
+    Newton's method started at m = target approaches the root monotonically from below."""
+    if target >= num:
+        raise ValueError("target unique count must be < number of rows")
+    lp = np.log1p(-zipf_pmf(num, alpha))
+    m = float(target)
+    for _ in range(100):
+        e = np.exp(m * lp)
+        f = float(np.sum(1.0 - e)) - target
+        df = float(-np.dot(lp, e))
+        step = -f / df
+        m += step
+        if abs(step) <= 1e-9 * m:
             break
-    return hi
+    return m
 
 
 def hotness(wl: Workload, m_unique: Optional[float] = None) -> np.ndarray:

@@ -242,3 +242,21 @@ def test_dlr_shaped_scaled_parity(torch_cuda):
         c.close()
     t.close()
     _TABLES.pop((wl.num_rows, wl.row_bytes), None)
+
+
+@pytest.mark.parametrize("ordered", [True, False])
+@pytest.mark.parametrize("host_sms", [1, 3, 16, 147])
+def test_host_range_ordering_parity(torch_cuda, ordered, host_sms):
+    """Large host bucket (>= kHostSortMin keys): range-ordered and unordered host reads
+    give the same bytes, for any number of host CTAs (intra-role barriers)."""
+    N, R = 300_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(5).permutation(N)]
+    t, (c,) = make_group(torch_cuda, N, R, 3000, 1, h)
+    c.set_host_ordering(ordered)
+    c.set_dedication(host_sms, 0)
+    keys = np.random.default_rng(6).integers(0, N, 40_000)
+    keys[::50] = -3
+    for _ in range(3):  # re-armed range counters across launches
+        per = check_batch(torch_cuda, c, t, keys, N, R, 1)
+        assert per[1] > 4096
+    c.close()
