@@ -76,7 +76,7 @@ class Clocks:
              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
         try:
-            self.p = subprocess.Popen(["nvidia-smi", f"--id={index}", f"--query-gpu={q}",
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={q}",
                                        "--format=csv,noheader,nounits", "-lms", "100"],
                                       stdout=self.f, stderr=subprocess.DEVNULL)
         except Exception:
@@ -141,7 +141,7 @@ def setup_table(wl, rank, ws, torch_dist):
         table = synth.HostTable(wl.num_rows, wl.row_bytes)
         table.fill()
     else:
-        path = f"/dev/shm/ugache_bench_{wl.name}_{os.getpid() if False else 'shared'}"
+        path = f"/dev/shm/ugache_bench_{wl.name}_{os.environ.get('MASTER_PORT', '0')}"
         if rank == 0:
             table = synth.HostTable(wl.num_rows, wl.row_bytes, shm_path=path, create=True)
             table.fill()
@@ -225,10 +225,18 @@ def main():
     rank, ws, local = dist_env()
     if ws != args.gpus:
         log(f"warning: --gpus {args.gpus} but WORLD_SIZE {ws}; using WORLD_SIZE")
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    ndev = torch.cuda.device_count()
+    dev_idx = local % ndev
+    torch.cuda.set_device(dev_idx)
+    dev = torch.device("cuda", dev_idx)
     if ws > 1:
-        tdist.init_process_group("nccl", device_id=dev)
+        # NCCL when every rank owns a GPU (the normal case); gloo only for the control plane
+        # when ranks share a device (a functional multi-rank run on a 1-GPU box).
+        if ndev >= ws:
+            tdist.init_process_group("nccl", device_id=dev)
+        else:
+            tdist.init_process_group("gloo")
+    local = dev_idx
 
     table = setup_table(wl, rank, ws, tdist)
     t0 = time.time()
@@ -282,7 +290,7 @@ def main():
     stream.synchronize()
     ugdist.barrier()
     torch.cuda.synchronize()
-    clocks = Clocks(local) if rank == 0 else None
+    clocks = Clocks(local) if rank == 0 else None  # samples every GPU of the node
     time.sleep(0.3 if clocks else 0)
     evs, loc_ms, gat_ms, per_src = [], [], [], []
     launches = 0
@@ -431,8 +439,11 @@ def main():
     if rank == 0:
         print(json.dumps(line), flush=True)
     cache.close()
+    ugdist.barrier()
     table.close()
     if ws > 1:
+        if rank == 0 and table.shm_path and os.path.exists(table.shm_path):
+            os.unlink(table.shm_path)
         tdist.destroy_process_group()
 
 

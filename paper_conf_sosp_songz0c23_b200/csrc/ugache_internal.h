@@ -17,10 +17,12 @@ constexpr int kDefaultHostSms = 8;
 // Default model bandwidths (bytes/s) when the caller passes 0 (R11):
 //  local = MEASURED_PEAKS.json hbm_gbs (STREAM-style copy on this pool's B200s),
 //  peer  = measured B200 peer copy per direction (B200_PROFILING.md: 770 GB/s),
-//  host  = pinned H2D cudaMemcpy on the B200 box (PCIe Gen5 x16, probe: 55.6 GB/s).
+//  host  = calibrated zero-copy throughput of random 512-B host rows with range-ordered
+//          reads on the B200 box (tools/calibrate.py, gnn_pa: 34.4 GB/s; the sequential
+//          pinned-H2D DMA peak is 55.6 GB/s).
 constexpr double kDefaultBwLocal = 6457.7e9;
 constexpr double kDefaultBwPeer = 770e9;
-constexpr double kDefaultBwHost = 55.6e9;
+constexpr double kDefaultBwHost = 34.4e9;
 
 struct Params {
   int S, host_sms, peer_sms;

@@ -65,7 +65,7 @@ def test_solve_rejects_nan_hotness_and_oversubscribed_sms():
 def _platform(cfg, plan):
     return Platform(G=cfg.num_gpus, row_bytes=cfg.row_bytes,
                     bw_local=cfg.bw_local or 6457.7e9, bw_peer=cfg.bw_peer or 770e9,
-                    bw_host=cfg.bw_host or 55.6e9, host_sms=plan.host_sms,
+                    bw_host=cfg.bw_host or 34.4e9, host_sms=plan.host_sms,
                     peer_sms=plan.peer_sms, num_sms=plan.num_sms)
 
 
