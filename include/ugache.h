@@ -163,9 +163,11 @@ ugache_status ugache_fill(ugache_ctx *ctx, void *stream);
  * key order P:626-627).  keys: n keys of key_type, device or host memory.  out: n*R bytes,
  * device or host memory, 16-byte aligned.  Device buffers: fully asynchronous on stream,
  * no host synchronisation, no collective; keys/out must stay valid until the stream
- * reaches the work.  Host buffers: staged through ctx-owned device buffers with async
- * copies on the same stream (the caller synchronises the stream before reading out).
- * n == 0: no work.  Requires ugache_fill and, for G > 1, peers (else ESTATE). */
+ * reaches the work.  Pinned (page-locked) host buffers: read / written in place by the
+ * kernels over PCIe (zero-copy; UGACHE_OPT_STAGE_HOST_IO = 1 stages them instead).
+ * Pageable host buffers: staged through ctx-owned device buffers with async copies on the
+ * same stream.  With any host buffer the caller synchronises the stream before reading
+ * out.  n == 0: no work.  Requires ugache_fill and, for G > 1, peers (else ESTATE). */
 ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type, uint64_t n,
                              void *out, void *stream);
 
@@ -176,11 +178,21 @@ ugache_status ugache_set_dedication(ugache_ctx *ctx, int32_t host_sms, int32_t p
 /* ugache_mode; FACTORED by default. */
 ugache_status ugache_set_mode(ugache_ctx *ctx, int32_t mode);
 
-/* Host-source read order (B200 box property): when on (default),
- * the host CTAs of the factored gather first order the host bucket by key range so the
- * rows in flight cover a small window of host address space, then copy in that order.
- * off = copy in bucket order.  Output is identical either way. */
-ugache_status ugache_set_host_ordering(ugache_ctx *ctx, int32_t on);
+/* Tuning options (ugache_set_option); none changes the output bytes.
+ *  UGACHE_OPT_HOST_ORDERING (default 1): the host CTAs of the factored gather first order
+ *    the host bucket by key range so the rows in flight cover a small window of host
+ *    address space (translation reach of the host aperture), then copy
+ *    in that order; 0 = copy in bucket order.
+ *  UGACHE_OPT_STAGE_HOST_IO (default 0): 1 = stage pinned host keys/out through device
+ *    buffers + cudaMemcpyAsync instead of zero-copy access from the kernels.
+ *  UGACHE_OPT_HOST_WARPS (default 8, 1..16): warps per host CTA that read host rows; the
+ *    others pad local work (A0 calibration knob). */
+typedef enum {
+  UGACHE_OPT_HOST_ORDERING = 0,
+  UGACHE_OPT_STAGE_HOST_IO = 1,
+  UGACHE_OPT_HOST_WARPS = 2
+} ugache_option;
+ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value);
 
 /* Per-source key counts of the last extract: per_source[j] for GPU j (j == rank: local),
  * per_source[G] for host (G+1 entries); bad_keys: out-of-range keys.  Synchronises with

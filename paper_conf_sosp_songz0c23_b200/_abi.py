@@ -24,6 +24,7 @@ POLICIES = {"ugache": POLICY_UGACHE, "replication": POLICY_REPLICATION,
             "partition": POLICY_PARTITION}
 KEY_I64, KEY_U32 = 0, 1
 MODE_FACTORED, MODE_RANDOM_DISPATCH = 0, 1
+OPT_HOST_ORDERING, OPT_STAGE_HOST_IO, OPT_HOST_WARPS = 0, 1, 2
 
 
 class ugache_config(ctypes.Structure):
@@ -73,7 +74,7 @@ SIGNATURES = {
     "ugache_extract": (_ST, [_P, _P, _c.c_int32, _c.c_uint64, _P, _P]),
     "ugache_set_dedication": (_ST, [_P, _c.c_int32, _c.c_int32]),
     "ugache_set_mode": (_ST, [_P, _c.c_int32]),
-    "ugache_set_host_ordering": (_ST, [_P, _c.c_int32]),
+    "ugache_set_option": (_ST, [_P, _c.c_int32, _c.c_int64]),
     "ugache_last_batch_stats": (_ST, [_P, _P, ctypes.POINTER(_c.c_uint64)]),
     "ugache_enable_timing": (_ST, [_P, _c.c_int32]),
     "ugache_last_batch_timing": (_ST, [_P, ctypes.POINTER(_c.c_float), ctypes.POINTER(_c.c_float)]),

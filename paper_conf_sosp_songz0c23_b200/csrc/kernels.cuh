@@ -28,6 +28,7 @@ constexpr int kGatherThreads = 512;  // 16 warps; one CTA per SM (forced via sme
 constexpr int kGatherWarps = kGatherThreads / 32;
 constexpr int kRowsInFlight = 8;     // rows per warp per step (U)
 constexpr int kLocalChunk = 64;      // rows per local-cursor claim
+constexpr int kHostWarps = 8;        // warps per host CTA reading host rows (A0 calibration)
 constexpr uint32_t kFullMask = 0xFFFFFFFFu;
 constexpr int kMaxSmId = 256;        // role table size, indexed by %smid
 
@@ -85,6 +86,7 @@ struct GatherParams {
   uint32_t range_shift;            // range = row >> range_shift
   uint32_t n_ranges;               // <= kMaxRanges
   int32_t host_sort;               // 0 = read the host bucket in bucket order
+  int32_t host_warps;              // warps per host CTA that copy host rows (window size)
 };
 
 struct RandomParams {
@@ -308,6 +310,22 @@ __device__ __forceinline__ void block_exclusive_scan(const uint32_t *src, uint32
   __syncthreads();
 }
 
+// In-order copy of the range-ordered host bucket: warps claim U consecutive entries from a
+// shared cursor (next claim prefetched), so the rows in flight are the most recent claims.
+template <int U>
+__device__ __forceinline__ void host_copy_ordered(const GatherParams &p, uint32_t cnt, int lane) {
+  const uint8_t *base = p.base[p.num_src - 1];
+  uint32_t next = 0;
+  if (lane == 0) next = atomicAdd(&p.ctrl->host_cursor, (uint32_t)U);
+  next = __shfl_sync(kFullMask, next, 0);
+  while (next < cnt) {
+    const uint32_t e0 = next;
+    if (lane == 0) next = atomicAdd(&p.ctrl->host_cursor, (uint32_t)U);
+    next = __shfl_sync(kFullMask, next, 0);
+    copy_rows<U>(base, p.out, p.row_bytes, p.host_sorted + e0, (int)min((uint32_t)U, cnt - e0), lane);
+  }
+}
+
 // Host role with range ordering: histogram -> barrier -> scan -> scatter -> barrier ->
 // dynamic in-order copy.  All host CTAs cooperate; `h`/`H` = index/count within the role.
 __device__ __forceinline__ void host_role_sorted(const GatherParams &p, const uint64_t *b,
@@ -336,17 +354,8 @@ __device__ __forceinline__ void host_role_sorted(const GatherParams &p, const ui
       p.range_cursor[i] = 0;
     }
   }
-  const uint8_t *base = p.base[p.num_src - 1];
-  uint32_t next = 0;
-  if (lane == 0) next = atomicAdd(&p.ctrl->host_cursor, (uint32_t)kRowsInFlight);
-  next = __shfl_sync(kFullMask, next, 0);
-  while (next < cnt) {
-    const uint32_t e0 = next;
-    if (lane == 0) next = atomicAdd(&p.ctrl->host_cursor, (uint32_t)kRowsInFlight);
-    next = __shfl_sync(kFullMask, next, 0);
-    copy_rows<kRowsInFlight>(base, p.out, p.row_bytes, p.host_sorted + e0,
-                             (int)min((uint32_t)kRowsInFlight, cnt - e0), lane);
-  }
+  if ((tid >> 5) >= p.host_warps) return;  // window control: the other warps pad local work
+  host_copy_ordered<kRowsInFlight>(p, cnt, lane);
 }
 
 // ---------------------------------------------------------------------------- K2

@@ -7,6 +7,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <mutex>
@@ -49,6 +50,8 @@ struct ugache_ctx {
   uint32_t *d_ranges = nullptr;  // 2 * kMaxRanges counters
   uint32_t range_shift = 0, n_ranges = 1;
   int host_sort = 1;
+  int host_warps = ugk::kHostWarps;  // env UGACHE_HOST_WARPS (A0 calibration knob)
+  int stage_host_io = 0;             // env UGACHE_STAGE_HOST_IO=1: stage pinned host I/O too
   std::vector<int> smids;  // sorted %smid values of the device (one per SM)
   // dedication / mode
   int host_sms = 0, peer_sms = 0;
@@ -104,6 +107,23 @@ bool is_device_pointer(const void *p, int *device) {
     return true;
   }
   return false;
+}
+
+enum class MemKind { kDevice, kPinned, kPageable };
+
+// Where a caller buffer lives; for pinned host memory also its device-mapped address.
+MemKind mem_kind(const void *p, void **mapped) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    (void)cudaGetLastError();
+    return MemKind::kPageable;
+  }
+  if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) return MemKind::kDevice;
+  if (a.type == cudaMemoryTypeHost && a.devicePointer) {
+    *mapped = a.devicePointer;
+    return MemKind::kPinned;
+  }
+  return MemKind::kPageable;
 }
 
 bool is_pinned_host(const void *p) {
@@ -263,6 +283,8 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   ctx->range_shift = 0;
   while (((N - 1) >> ctx->range_shift) + 1 > (uint64_t)ugk::kMaxRanges) ++ctx->range_shift;
   ctx->n_ranges = (uint32_t)(((N - 1) >> ctx->range_shift) + 1);
+  if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_HOST_WARPS")) ctx->host_warps = std::max(1, std::min(ugk::kGatherWarps, atoi(e)));
   for (int i = 0; i < 3; ++i) UG_CUDA(ctx, cudaEventCreate(&ctx->ev[i]));
   ctx->src_base[cfg->rank] = ctx->slab;
   ctx->src_base[G] = ctx->host_table_dev;
@@ -503,10 +525,17 @@ ugache_status ugache_set_mode(ugache_ctx *ctx, int32_t mode) {
   return UGACHE_OK;
 }
 
-ugache_status ugache_set_host_ordering(ugache_ctx *ctx, int32_t on) {
+ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value) {
   if (!ctx) return UGACHE_EINVAL;
-  ctx->host_sort = on != 0;
-  return UGACHE_OK;
+  switch (option) {
+    case UGACHE_OPT_HOST_ORDERING: ctx->host_sort = value != 0; return UGACHE_OK;
+    case UGACHE_OPT_STAGE_HOST_IO: ctx->stage_host_io = value != 0; return UGACHE_OK;
+    case UGACHE_OPT_HOST_WARPS:
+      if (value < 1 || value > ugk::kGatherWarps) return UGACHE_EINVAL;
+      ctx->host_warps = (int)value;
+      return UGACHE_OK;
+  }
+  return UGACHE_EINVAL;
 }
 
 ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type, uint64_t n,
@@ -526,22 +555,33 @@ ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type
   const uint32_t R = ctx->cfg.row_bytes;
   const size_t key_bytes = key_type == UGACHE_KEY_I64 ? 8 : 4;
 
+  // Host buffers: pinned (page-locked, mapped) ones are read / written in place by the
+  // kernels over PCIe -- the H2D of the keys and the D2H of the rows are fused into the
+  // locate and gather kernels; pageable ones are staged through ctx-owned device buffers.
   const void *dkeys = keys;
-  if (!is_device_pointer(keys, nullptr)) {
+  void *mapped = nullptr;
+  const MemKind kkind = mem_kind(keys, &mapped);
+  if (kkind == MemKind::kPinned && !ctx->stage_host_io) {
+    dkeys = mapped;
+  } else if (kkind != MemKind::kDevice) {
     st = ensure_stage(ctx, &ctx->d_keys_stage, &ctx->keys_stage_bytes, n * key_bytes);
     if (st != UGACHE_OK) return st;
     UG_CUDA(ctx, cudaMemcpyAsync(ctx->d_keys_stage, keys, n * key_bytes, cudaMemcpyHostToDevice, s));
     dkeys = ctx->d_keys_stage;
   }
   uint8_t *dout = static_cast<uint8_t *>(out);
-  const bool host_out = !is_device_pointer(out, nullptr);
-  if (host_out) {
+  const MemKind okind = mem_kind(out, &mapped);
+  const bool staged_out = okind == MemKind::kPageable || (okind == MemKind::kPinned && ctx->stage_host_io);
+  if (staged_out) {
     st = ensure_stage(ctx, &ctx->d_out_stage, &ctx->out_stage_bytes, n * (size_t)R);
     if (st != UGACHE_OK) return st;
     dout = static_cast<uint8_t *>(ctx->d_out_stage);
-  } else if (reinterpret_cast<uintptr_t>(out) % 16 != 0) {
-    return fail(ctx, UGACHE_EINVAL, "out must be 16-byte aligned");
+  } else {
+    if (okind == MemKind::kPinned) dout = static_cast<uint8_t *>(mapped);
+    if (reinterpret_cast<uintptr_t>(dout) % 16 != 0)
+      return fail(ctx, UGACHE_EINVAL, "out must be 16-byte aligned");
   }
+  const bool host_out = staged_out;
 
   if (ctx->mode == UGACHE_MODE_RANDOM_DISPATCH) {
     ugk::RandomParams rp;
@@ -600,6 +640,7 @@ ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type
     gp.range_shift = ctx->range_shift;
     gp.n_ranges = ctx->n_ranges;
     gp.host_sort = ctx->host_sort;
+    gp.host_warps = ctx->host_warps;
     int grid = 0;
     build_roles(ctx, &gp, &grid);
     void *kargs[] = {&gp};

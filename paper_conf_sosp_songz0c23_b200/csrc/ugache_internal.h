@@ -13,7 +13,7 @@ constexpr int kMaxSrc = UGACHE_MAX_GPUS + 1;
 constexpr int kDefaultNumSms = 148;
 // Default core dedication for host extraction: "a small number of cores for host"
 // (P:1211-1213).  Set from the A0 calibration on B200 (DESIGN.md section "calibration").
-constexpr int kDefaultHostSms = 8;
+constexpr int kDefaultHostSms = 12;
 // Default model bandwidths (bytes/s) when the caller passes 0 (R11):
 //  local = MEASURED_PEAKS.json hbm_gbs (STREAM-style copy on this pool's B200s),
 //  peer  = measured B200 peer copy per direction (B200_PROFILING.md: 770 GB/s),

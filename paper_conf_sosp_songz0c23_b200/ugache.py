@@ -136,8 +136,14 @@ class UGache:
         m = {"factored": _abi.MODE_FACTORED, "random": _abi.MODE_RANDOM_DISPATCH}[mode]
         check(lib().ugache_set_mode(self.ctx, m), "ugache_set_mode", self.ctx)
 
+    def set_option(self, option: int, value: int):
+        check(lib().ugache_set_option(self.ctx, option, int(value)), "ugache_set_option", self.ctx)
+
     def set_host_ordering(self, on: bool):
-        check(lib().ugache_set_host_ordering(self.ctx, int(on)), "ugache_set_host_ordering", self.ctx)
+        self.set_option(_abi.OPT_HOST_ORDERING, int(on))
+
+    def set_stage_host_io(self, on: bool):
+        self.set_option(_abi.OPT_STAGE_HOST_IO, int(on))
 
     def enable_timing(self, on: bool = True):
         check(lib().ugache_enable_timing(self.ctx, int(on)), "ugache_enable_timing", self.ctx)

@@ -252,7 +252,7 @@ def test_host_range_ordering_parity(torch_cuda, ordered, host_sms):
     N, R = 300_000, 512
     h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(5).permutation(N)]
     t, (c,) = make_group(torch_cuda, N, R, 3000, 1, h)
-    c.set_host_ordering(ordered)
+    c.set_host_ordering(ordered)  # UGACHE_OPT_HOST_ORDERING
     c.set_dedication(host_sms, 0)
     keys = np.random.default_rng(6).integers(0, N, 40_000)
     keys[::50] = -3
@@ -260,3 +260,26 @@ def test_host_range_ordering_parity(torch_cuda, ordered, host_sms):
         per = check_batch(torch_cuda, c, t, keys, N, R, 1)
         assert per[1] > 4096
     c.close()
+
+
+@pytest.mark.parametrize("staged", [False, True])
+def test_pinned_host_io_zero_copy_and_staged(torch_cuda, staged):
+    """Pinned host keys/out are used in place by the kernels (default) or staged; both
+    produce the oracle's bytes, including zero rows of out-of-range keys."""
+    N, R = 200_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(8).permutation(N)]
+    t, group = make_group(torch_cuda, N, R, 4000, 2, h)
+    keys = np.random.default_rng(9).integers(0, N, 30_000)
+    keys[::97] = N + 1
+    pk = torch_cuda.from_numpy(keys).pin_memory()
+    for g, c in enumerate(group):
+        c.set_stage_host_io(staged)
+        out = torch_cuda.full((len(keys), R), 7, dtype=torch_cuda.uint8).pin_memory()
+        c.extract(pk, out)
+        torch_cuda.cuda.synchronize()
+        ref, bad = oracle.gather(t.ptr, N, R, keys)
+        assert np.array_equal(out.numpy(), ref)
+        per, nbad = c.last_batch_stats()
+        assert nbad == bad
+    for c in group:
+        c.close()

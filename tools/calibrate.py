@@ -25,6 +25,7 @@ def main():
     ap.add_argument("--reps", type=int, default=6)
     ap.add_argument("--order", default="1,0")
     ap.add_argument("--random", action="store_true")
+    ap.add_argument("--combos", default="", help="rows:warps,... (UGACHE_HOST_ROWS/WARPS per ctx)")
     args = ap.parse_args()
     import torch
     import synth
@@ -40,16 +41,37 @@ def main():
     cfg = make_config(wl.num_rows, wl.row_bytes, wl.capacity_rows)
     plan, order = solve(cfg, h)
     del h
-    cache = UGache(table, wl.num_rows, wl.row_bytes, wl.capacity_rows, plan=plan, order=order)
-    del order
-    cache.fill()
-    torch.cuda.synchronize()
+    def new_cache():
+        c = UGache(table, wl.num_rows, wl.row_bytes, wl.capacity_rows, plan=plan, order=order)
+        c.fill()
+        torch.cuda.synchronize()
+        c.enable_timing(True)
+        return c
+
+    combos = [tuple(int(v) for v in c.split(":")) for c in args.combos.split(",") if c]
+    cache = new_cache()
     batches = [torch.from_numpy(synth.make_batch(wl, 0, i)).cuda() for i in range(2)]
     n = batches[0].numel()
     out = torch.empty((n, wl.row_bytes), dtype=torch.uint8, device="cuda")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     cache.enable_timing(True)
     res = []
+    for rows, warps in combos:
+        os.environ["UGACHE_HOST_ROWS"] = str(rows)
+        os.environ["UGACHE_HOST_WARPS"] = str(warps)
+        c2 = new_cache()
+        for hs in [int(x) for x in args.host_sms.split(",")]:
+            c2.set_dedication(hs, 0)
+            gms = []
+            for r in range(args.reps + 1):
+                flush.fill_(r)
+                c2.extract(batches[r % 2], out)
+                a, b = c2.last_batch_timing()
+                if r:
+                    gms.append(b)
+            rec = {"rows": rows, "warps": warps, "host_sms": hs, "gather_ms": statistics.median(gms)}
+            print(json.dumps(rec), flush=True)
+        c2.close()
     for ordered in [int(x) for x in args.order.split(",")]:
         cache.set_host_ordering(bool(ordered))
         for hs in [int(x) for x in args.host_sms.split(",")]:
@@ -79,8 +101,9 @@ def main():
             if r:
                 gms.append(b)
         print(json.dumps({"mode": "random", "gather_ms": statistics.median(gms)}), flush=True)
-    best = min(res, key=lambda x: x["gather_ms"])
-    print(json.dumps({"best": best}), flush=True)
+    if res:
+        best = min(res, key=lambda x: x["gather_ms"])
+        print(json.dumps({"best": best}), flush=True)
 
 
 if __name__ == "__main__":
