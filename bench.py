@@ -57,6 +57,9 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--no-verify", action="store_true")
     ap.add_argument("--extra", action="store_true", help="also time the random-dispatch ablation")
+    ap.add_argument("--no-clocks", action="store_true", help="do not sample nvidia-smi (diagnostics only)")
+    ap.add_argument("--host-tier", action="store_true",
+                    help="read host rows from a hotness-ordered pinned copy (UGACHE_FLAG_HOST_TIER)")
     return ap.parse_args()
 
 
@@ -202,6 +205,7 @@ def config_dict(args, wl, ws):
             "keys_per_batch_per_gpu": wl.keys_per_batch, "batch_kind": wl.batch_kind,
             "alpha": wl.alpha, "cache_ratio": args.cache_ratio if args.cache_ratio is not None
             else wl.cache_ratio, "policy": args.policy, "mode": args.mode,
+            "host_tier": bool(getattr(args, "host_tier", False)),
             "parallelism": f"dp{ws}",
             "l2": "256 MiB L2-flush write between timed steps (outside the events); per-step "
                   "output > L2"}
@@ -250,9 +254,22 @@ def main():
     log(f"solve in {time.time() - t0:.1f}s: k={plan.k} band_end={plan.band_end} z={plan.z:.3e}")
     del h
     t0 = time.time()
+    tier = False
+    if args.host_tier:
+        tier = True  # N = 1: the ctx builds its own rank-ordered host tier
+        if ws > 1:   # one tier per node in /dev/shm, filled by rank 0, mapped by all
+            from paper_conf_sosp_songz0c23_b200 import fill_host_tier, host_tier_rows
+            trows = host_tier_rows(plan, wl.num_rows)
+            tpath = f"/dev/shm/ugache_tier_{wl.name}_{os.environ.get('MASTER_PORT', '0')}"
+            if rank == 0:
+                tier = synth.HostTable(max(trows, 1), wl.row_bytes, shm_path=tpath, create=True)
+                fill_host_tier(cfg, order, plan, table, tier)
+            tdist.barrier()
+            if rank != 0:
+                tier = synth.HostTable(max(trows, 1), wl.row_bytes, shm_path=tpath, create=False)
     cache = UGache(table, wl.num_rows, wl.row_bytes, C, num_gpus=ws, rank=rank, device=local,
                    policy=args.policy, plan=plan, order=order, host_sms=args.host_sms,
-                   peer_sms=args.peer_sms)
+                   peer_sms=args.peer_sms, host_tier=tier)
     log(f"init (register host table, location table, slab) in {time.time() - t0:.1f}s")
     ugdist.connect(cache, order=order)
     del order
@@ -290,7 +307,7 @@ def main():
     stream.synchronize()
     ugdist.barrier()
     torch.cuda.synchronize()
-    clocks = Clocks(local) if rank == 0 else None  # samples every GPU of the node
+    clocks = Clocks(local) if (rank == 0 and not args.no_clocks) else None  # every GPU of the node
     time.sleep(0.3 if clocks else 0)
     evs, loc_ms, gat_ms, per_src = [], [], [], []
     launches = 0
@@ -306,6 +323,7 @@ def main():
     torch.cuda.synchronize()
     ugdist.barrier()
     clk = clocks.stop() if clocks else None
+    log("per-step gather ms: " + " ".join(f"{x:.3f}" for x in gat_ms))
     step_ms = [s.elapsed_time(e) for s, e in evs]
     my_total_s = sum(step_ms) / 1e3
     max_total_s = ugdist.max_over_ranks(my_total_s)
@@ -486,10 +504,13 @@ def main():
         print(json.dumps(line), flush=True)
     cache.close()
     ugdist.barrier()
-    table.close()
+    for buf in (table, tier):
+        if isinstance(buf, synth.HostTable):
+            path = buf.shm_path
+            buf.close()
+            if ws > 1 and rank == 0 and path and os.path.exists(path):
+                os.unlink(path)
     if ws > 1:
-        if rank == 0 and table.shm_path and os.path.exists(table.shm_path):
-            os.unlink(table.shm_path)
         tdist.destroy_process_group()
 
 

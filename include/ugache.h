@@ -38,7 +38,8 @@ extern "C" {
 #define UGACHE_VERSION 1
 #define UGACHE_MAX_GPUS 16
 /* Location-table entry: (src << 56) | row.  src = j < G: GPU j's cache slab, row = slot;
- * src = G: host DRAM, row = key (the host holds every entry). */
+ * src = G: host DRAM, row = key (the host holds every entry), or the host-tier
+ * slot when UGACHE_FLAG_HOST_TIER is set. */
 #define UGACHE_LOC_SRC_SHIFT 56
 #define UGACHE_LOC_ROW_MASK ((((uint64_t)1) << 56) - 1)
 
@@ -84,8 +85,15 @@ typedef struct {
   int32_t host_sms;       /* SMs dedicated to host extraction; 0 = default  */
   int32_t peer_sms;       /* SMs dedicated to each peer; 0 = floor((S-host)/(G-1)) */
   int32_t num_sms;        /* S; 0 = the device's SM count (148 on B200)                   */
-  int32_t flags;          /* must be 0                                                    */
+  int32_t flags;          /* UGACHE_FLAG_* bits; other bits must be 0                     */
 } ugache_config;
+
+/* Host tier (reading R24): the entries that no GPU caches (hotness
+ * ranks >= band_end) are read from a pinned host copy laid out in hotness-rank order
+ * instead of the caller's key-ordered table, so host reads concentrate in a dense prefix
+ * of host address space.  Location-table rows of the host source are then tier slots
+ * (slot t holds the key of rank band_end + t) instead of keys. */
+#define UGACHE_FLAG_HOST_TIER 1
 
 /* Solver output (section 6.2 model evaluated for the chosen placement). */
 typedef struct {
@@ -119,6 +127,15 @@ ugache_status ugache_build_placement(const ugache_config *cfg, const uint64_t *o
                                      const ugache_plan *plan, int32_t gpu, uint64_t *loc,
                                      uint64_t *slot_keys, uint64_t *n_slots);
 
+/* Host tier (UGACHE_FLAG_HOST_TIER): number of tier rows, N - band_end. */
+uint64_t ugache_host_tier_rows(const ugache_plan *plan, uint64_t num_rows);
+
+/* Fill a caller-provided host tier: tier[t*R ..) = table row order[band_end + t] for
+ * t < tier_rows (parallel host copy, no GPU).  tier: ugache_host_tier_rows * R bytes. */
+ugache_status ugache_fill_host_tier(const ugache_config *cfg, const uint64_t *order,
+                                    const ugache_plan *plan, const void *host_table,
+                                    void *tier);
+
 /* ---- context lifecycle -------------------------------------------------------------- */
 
 /* Create the ctx of GPU cfg->rank on device cfg->device: solve the placement, build this
@@ -131,10 +148,14 @@ ugache_status ugache_init(ugache_ctx **ctx, const ugache_config *cfg, const void
                           const float *hotness);
 
 /* Same as ugache_init but with a precomputed order/plan (every rank of a process group can
- * share one solve).  order: N entries; plan from ugache_solve with the same cfg. */
+ * share one solve).  order: N entries; plan from ugache_solve with the same cfg.
+ * host_tier: with UGACHE_FLAG_HOST_TIER, an optional caller-owned tier already filled by
+ * ugache_fill_host_tier (shared by the ranks of a node; pinned by the library unless
+ * already pinned; must outlive the ctx); NULL = the ctx builds and owns its own tier.
+ * ugache_init with the flag always builds its own. */
 ugache_status ugache_init_with_plan(ugache_ctx **ctx, const ugache_config *cfg,
                                     const void *host_table, const uint64_t *order,
-                                    const ugache_plan *plan);
+                                    const ugache_plan *plan, const void *host_tier);
 
 ugache_status ugache_get_plan(const ugache_ctx *ctx, ugache_plan *plan);
 
@@ -186,12 +207,22 @@ ugache_status ugache_set_mode(ugache_ctx *ctx, int32_t mode);
  *  UGACHE_OPT_STAGE_HOST_IO (default 0): 1 = stage pinned host keys/out through device
  *    buffers + cudaMemcpyAsync instead of zero-copy access from the kernels.
  *  UGACHE_OPT_HOST_WARPS (default 8, 1..16): warps per host CTA that read host rows; the
- *    others pad local work (A0 calibration knob). */
+ *    others pad local work (A0 calibration knob).
+ *  UGACHE_OPT_DEDICATION: UGACHE_DEDICATE_SMS = the paper's core dedication, whole SMs per
+ *    source; UGACHE_DEDICATE_WARPS = the same dedication at warp granularity:
+ *    on every SM, UGACHE_OPT_WARP_HOST warps serve the host and UGACHE_OPT_WARP_PEER warps
+ *    serve each peer, the others start on local rows.
+ *  UGACHE_OPT_WARP_HOST / UGACHE_OPT_WARP_PEER (default 1 / 1): warps per SM in
+ *    UGACHE_DEDICATE_WARPS mode; host + (G-1) * peer <= 16. */
 typedef enum {
   UGACHE_OPT_HOST_ORDERING = 0,
   UGACHE_OPT_STAGE_HOST_IO = 1,
-  UGACHE_OPT_HOST_WARPS = 2
+  UGACHE_OPT_HOST_WARPS = 2,
+  UGACHE_OPT_DEDICATION = 3,
+  UGACHE_OPT_WARP_HOST = 4,
+  UGACHE_OPT_WARP_PEER = 5
 } ugache_option;
+typedef enum { UGACHE_DEDICATE_SMS = 0, UGACHE_DEDICATE_WARPS = 1 } ugache_dedication;
 ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value);
 
 /* Per-source key counts of the last extract: per_source[j] for GPU j (j == rank: local),

@@ -84,7 +84,7 @@ def rank_order(h: Optional[np.ndarray], N: int) -> np.ndarray:
 
 
 # ----------------------------------------------------------------------------- policies
-def policy_placement(order: np.ndarray, N: int, C: int, G: int, k: int):
+def policy_placement(order: np.ndarray, N: int, C: int, G: int, k: int, host_tier: bool = False):
     """Hot-replicate / warm-partition placement with replicated prefix length k.
 
     * ranks [0, k): on every GPU ("every GPU caches the hottest entries", replication,
@@ -94,6 +94,9 @@ def policy_placement(order: np.ndarray, N: int, C: int, G: int, k: int):
     * the rest: host DRAM (fallback location).
     k = C is replication, k = 0 is partition, 0 < k < C is the hot-replicate /
     warm-partition family of ref [39].
+
+    host_tier (R24): the host rows live in a copy ordered by hotness rank, so a
+    host entry's row is its tier slot ``rank - band_end`` instead of its key.
 
     Returns (loc[G, N] uint64, slot_keys: list of G uint64 arrays)."""
     C = min(C, N)
@@ -107,6 +110,8 @@ def policy_placement(order: np.ndarray, N: int, C: int, G: int, k: int):
     slot_keys: List[np.ndarray] = []
     for g in range(G):
         lg = enc(G, np.arange(N))                       # default: host, row = key
+        if host_tier:                                   # host row = tier slot
+            lg[order[band_end:]] = enc(G, np.arange(N - band_end))
         lg[order[:k]] = enc(g, np.arange(k))            # replicated prefix, slot = rank
         lg[order[band]] = (owner.astype(np.uint64) << SRC_SHIFT) | slot.astype(np.uint64)
         loc[g] = lg
@@ -161,10 +166,12 @@ def solve_sweep(h: np.ndarray, N: int, C: int, plat: Platform):
 
 
 # ----------------------------------------------------------------------------- checker
-def check_placement(loc: np.ndarray, slot_keys: List[np.ndarray], N: int, C: int):
+def check_placement(loc: np.ndarray, slot_keys: List[np.ndarray], N: int, C: int,
+                    tier_keys: Optional[np.ndarray] = None):
     """Placement invariants (SURVEY.md section 8(c) checker items 1-4); raises AssertionError.
 
-    1. resolution: LT_g[k] = (host, k) or (GPU j, slot) with slot < n_slots_j and
+    1. resolution: LT_g[k] = (host, k) [or (host, t) with tier_keys[t] == k for a host
+       tier] or (GPU j, slot) with slot < n_slots_j and
        slot_keys_j[slot] == k  ("Each cached embedding entry is associated with its source
        location in the format of <GPU_i, Offset>", P:946-952);
     2. capacity: n_slots_j <= C  (sum_e s^e_j <= Cap_j, P:1346-1353);
@@ -182,7 +189,12 @@ def check_placement(loc: np.ndarray, slot_keys: List[np.ndarray], N: int, C: int
         keys = np.arange(N)
         assert np.all((src >= 0) & (src <= G)), f"GPU {g}: bad source id"
         host = src == G
-        assert np.all(row[host] == keys[host]), f"GPU {g}: host row != key"
+        if tier_keys is None:
+            assert np.all(row[host] == keys[host]), f"GPU {g}: host row != key"
+        else:  # host tier: tier slot row holds the key
+            tk = np.asarray(tier_keys, dtype=np.int64)
+            assert np.all(row[host] < len(tk)), f"GPU {g}: host tier slot out of range"
+            assert np.all(tk[row[host]] == keys[host]), f"GPU {g}: host tier slot holds another key"
         for j in range(G):
             m = src == j
             sk = np.asarray(slot_keys[j], dtype=np.int64)

@@ -9,6 +9,8 @@ The product is ``libugache.so`` (C ABI in ``include/ugache.h``, sm_100a kernels 
 * :mod:`.dist`   -- torch.distributed control plane (IPC-handle exchange, barriers);
 * :mod:`.build`  -- nvcc build of the library (sm_100a).
 """
-from .ugache import UGache, build_placement, connect_in_process, make_config, solve  # noqa: F401
+from .ugache import (UGache, build_placement, connect_in_process, fill_host_tier,  # noqa: F401
+                     host_tier_rows, make_config, solve)
 
-__all__ = ["UGache", "solve", "build_placement", "make_config", "connect_in_process"]
+__all__ = ["UGache", "solve", "build_placement", "make_config", "connect_in_process",
+           "fill_host_tier", "host_tier_rows"]

@@ -25,6 +25,9 @@ POLICIES = {"ugache": POLICY_UGACHE, "replication": POLICY_REPLICATION,
 KEY_I64, KEY_U32 = 0, 1
 MODE_FACTORED, MODE_RANDOM_DISPATCH = 0, 1
 OPT_HOST_ORDERING, OPT_STAGE_HOST_IO, OPT_HOST_WARPS = 0, 1, 2
+OPT_DEDICATION, OPT_WARP_HOST, OPT_WARP_PEER = 3, 4, 5
+DEDICATE_SMS, DEDICATE_WARPS = 0, 1
+FLAG_HOST_TIER = 1
 
 
 class ugache_config(ctypes.Structure):
@@ -63,7 +66,10 @@ SIGNATURES = {
                                      _c.c_int32, _P, _P, ctypes.POINTER(_c.c_uint64)]),
     "ugache_init": (_ST, [ctypes.POINTER(_P), ctypes.POINTER(ugache_config), _P, _P]),
     "ugache_init_with_plan": (_ST, [ctypes.POINTER(_P), ctypes.POINTER(ugache_config), _P, _P,
-                                    ctypes.POINTER(ugache_plan)]),
+                                    ctypes.POINTER(ugache_plan), _P]),
+    "ugache_host_tier_rows": (_c.c_uint64, [ctypes.POINTER(ugache_plan), _c.c_uint64]),
+    "ugache_fill_host_tier": (_ST, [ctypes.POINTER(ugache_config), _P, ctypes.POINTER(ugache_plan),
+                                    _P, _P]),
     "ugache_get_plan": (_ST, [_P, ctypes.POINTER(ugache_plan)]),
     "ugache_slab": (_ST, [_P, ctypes.POINTER(_P), ctypes.POINTER(_c.c_uint64),
                           ctypes.POINTER(_c.c_uint64)]),

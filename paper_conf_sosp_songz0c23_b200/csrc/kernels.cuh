@@ -50,7 +50,8 @@ struct Ctrl {
 // key-range order so that the rows in flight span a small window of host address space
 // (IOMMU/ATS translation reach), instead of the whole table.
 constexpr int kMaxRanges = 4096;
-constexpr uint32_t kHostSortMin = 4096;  // below this many host keys, read unordered
+constexpr uint32_t kHostSortMin = 4096;  // never order fewer host keys than this
+constexpr int kRowsPerSmRound = kGatherWarps * kRowsInFlight;  // rows one SM keeps in flight
 
 struct LocateParams {
   const void *keys;
@@ -74,11 +75,15 @@ struct GatherParams {
   uint32_t row_bytes;
   int32_t num_src;
   int32_t local_src;
-  int32_t n_roles;
-  int32_t role_src[kMaxSrc];       // role r serves source role_src[r]
-  int32_t role_count[kMaxSrc];     // number of SMs (= CTAs) with role r
-  uint8_t sm_role[kMaxSmId];       // role of the CTA running on SM %smid
-  uint8_t sm_role_idx[kMaxSmId];   // its index within the role
+  // core dedication, resolved per launch on the device from the counts
+  int32_t num_sms;
+  int32_t host_sms;                // calibrated host SMs (dense host bucket)
+  int32_t host_sms_max;            // cap for a sparse host bucket (S - peers' SMs)
+  int32_t peer_sms;                // SMs per peer
+  int32_t n_peers;                 // G - 1
+  int32_t peer_src[kMaxSrc];       // the peer GPU ids, in role order
+  uint32_t host_sort_min;          // host keys needed for range-ordered reads
+  uint8_t sm_pos[kMaxSmId];        // position of SM %smid in the chip-spreading order
   // host range ordering
   uint64_t *host_sorted;           // bucket_cap entries of scratch
   uint32_t *range_count;           // kMaxRanges, zero between launches
@@ -86,7 +91,10 @@ struct GatherParams {
   uint32_t range_shift;            // range = row >> range_shift
   uint32_t n_ranges;               // <= kMaxRanges
   int32_t host_sort;               // 0 = read the host bucket in bucket order
-  int32_t host_warps;              // warps per host CTA that copy host rows (window size)
+  int32_t host_warps;              // SM mode: warps per host CTA copying host rows;
+                                   // warp mode: host warps on every SM
+  int32_t peer_warps;              // warp mode: warps per peer on every SM
+  int32_t warp_dedication;         // 0 = SM-granular roles (paper), 1 = warp-granular roles
 };
 
 struct RandomParams {
@@ -326,11 +334,11 @@ __device__ __forceinline__ void host_copy_ordered(const GatherParams &p, uint32_
   }
 }
 
-// Host role with range ordering: histogram -> barrier -> scan -> scatter -> barrier ->
-// dynamic in-order copy.  All host CTAs cooperate; `h`/`H` = index/count within the role.
-__device__ __forceinline__ void host_role_sorted(const GatherParams &p, const uint64_t *b,
-                                                 uint32_t cnt, int h, int H, uint32_t *s_tab) {
-  const int tid = threadIdx.x, lane = tid & 31;
+// Range ordering of the host bucket into p.host_sorted: histogram -> barrier -> scan ->
+// scatter -> barrier.  CTAs h = 0..H-1 cooperate with all their threads.
+__device__ __forceinline__ void host_order(const GatherParams &p, const uint64_t *b,
+                                           uint32_t cnt, int h, int H, uint32_t *s_tab) {
+  const int tid = threadIdx.x;
   const uint32_t lo = (uint32_t)((uint64_t)cnt * h / H), hi = (uint32_t)((uint64_t)cnt * (h + 1) / H);
   for (uint32_t i = tid; i < p.n_ranges; i += blockDim.x) s_tab[i] = 0;
   __syncthreads();
@@ -354,8 +362,23 @@ __device__ __forceinline__ void host_role_sorted(const GatherParams &p, const ui
       p.range_cursor[i] = 0;
     }
   }
-  if ((tid >> 5) >= p.host_warps) return;  // window control: the other warps pad local work
-  host_copy_ordered<kRowsInFlight>(p, cnt, lane);
+}
+
+// Host role (SM-granular dedication) with range ordering: the host CTAs order the bucket,
+// then `host_warps` warps of each copy rows in order; the other warps pad local work.
+__device__ __forceinline__ void host_role_sorted(const GatherParams &p, const uint64_t *b,
+                                                 uint32_t cnt, int h, int H, uint32_t *s_tab) {
+  host_order(p, b, cnt, h, H, s_tab);
+  if ((int)(threadIdx.x >> 5) >= p.host_warps) return;  // window control
+  host_copy_ordered<kRowsInFlight>(p, cnt, threadIdx.x & 31);
+}
+
+// Static warp striding of W warps (this one = gw) over a bucket of cnt rows of one source.
+__device__ __forceinline__ void stride_copy(const GatherParams &p, const uint64_t *b, uint32_t cnt,
+                                            const uint8_t *base, uint32_t gw, uint32_t W, int lane) {
+  for (uint32_t e0 = gw * kRowsInFlight; e0 < cnt; e0 += W * kRowsInFlight)
+    copy_rows<kRowsInFlight>(base, p.out, p.row_bytes, b + e0,
+                             (int)min((uint32_t)kRowsInFlight, cnt - e0), lane);
 }
 
 // ---------------------------------------------------------------------------- K2
@@ -364,29 +387,61 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
   extern __shared__ __align__(16) uint32_t s_dyn[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   // Role of this CTA = role of the SM it runs on (one CTA per SM, cooperative launch):
-  // the B200 replacement of the paper's MPS core limits.
+  // the B200 replacement of the paper's MPS core limits.  SMs are taken in
+  // the order of a chip-spreading permutation (sm_pos): [host | peer_0 | ... | local].
   uint32_t smid;
   asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-  const int r = smid < (uint32_t)kMaxSmId ? p.sm_role[smid] : p.n_roles - 1;
-  const int my_src = p.role_src[r];
-  const int my_idx = smid < (uint32_t)kMaxSmId ? p.sm_role_idx[smid] : 0;
-  const int role_ctas = p.role_count[r];
+  const int pos = smid < (uint32_t)kMaxSmId ? p.sm_pos[smid] : p.num_sms - 1;
+  const int host_src = p.num_src - 1;
+  const uint32_t n_host = p.ctrl->counts[host_src];
+  const bool host_dense = p.host_sort && n_host >= p.host_sort_min;
   const uint32_t R = p.row_bytes;
 
-  const int host_src = p.num_src - 1;
-  if (my_src == host_src && p.host_sort && p.ctrl->counts[host_src] >= kHostSortMin) {
-    host_role_sorted(p, p.buckets + (uint64_t)host_src * p.bucket_cap, p.ctrl->counts[host_src],
-                     my_idx, role_ctas, s_dyn);
+  if (p.warp_dedication) {
+    // Warp-granular dedication: on EVERY SM, warps [0, hw) serve the
+    // host and the next pw warps each peer; the rest start on local work.  Concurrency per
+    // slow source stays bounded (S*hw or S*pw warps) while the requests come from all GPCs
+    // and no SM idles behind a slow link.
+    const int S = p.num_sms, hw = p.host_warps, pw = p.peer_warps;
+    const uint64_t *bh = p.buckets + (uint64_t)host_src * p.bucket_cap;
+    if (host_dense) host_order(p, bh, n_host, pos, S, s_dyn);
+    if (warp < hw) {
+      if (host_dense) host_copy_ordered<kRowsInFlight>(p, n_host, lane);
+      else stride_copy(p, bh, n_host, p.base[host_src], (uint32_t)(pos * hw + warp), (uint32_t)(S * hw), lane);
+    } else if (warp < hw + p.n_peers * pw) {
+      const int j = p.peer_src[(warp - hw) / pw];
+      stride_copy(p, p.buckets + (uint64_t)j * p.bucket_cap, p.ctrl->counts[j], p.base[j],
+                  (uint32_t)(pos * pw + (warp - hw) % pw), (uint32_t)(S * pw), lane);
+    }
+  } else {
+  // Host SMs: the calibrated count when the host bucket is dense enough for ordered reads
+  // (throughput-bound); otherwise enough SMs to put the whole bucket in flight in about one
+  // round (latency-bound), capped so every peer keeps its dedicated SMs.  Every CTA derives
+  // the same split from the same counts.
+  int H = p.host_sms;
+  if (!host_dense)
+    H = max(H, min(p.host_sms_max, (int)((n_host + kRowsPerSmRound - 1) / kRowsPerSmRound)));
+  int my_src, my_idx, role_ctas;
+  if (pos < H) {
+    my_src = host_src, my_idx = pos, role_ctas = H;
+  } else if (pos - H < p.n_peers * p.peer_sms) {
+    my_src = p.peer_src[(pos - H) / p.peer_sms];
+    my_idx = (pos - H) % p.peer_sms, role_ctas = p.peer_sms;
+  } else {
+    my_src = p.local_src, my_idx = 0, role_ctas = 0;
+  }
+
+  if (my_src == host_src && host_dense) {
+    host_role_sorted(p, p.buckets + (uint64_t)host_src * p.bucket_cap, n_host, my_idx, role_ctas,
+                     s_dyn);
   } else if (my_src != p.local_src) {
     // dedicated non-local extraction: static warp striding over this source's bucket
     const uint32_t cnt = p.ctrl->counts[my_src];
     const uint64_t *b = p.buckets + (uint64_t)my_src * p.bucket_cap;
     const uint8_t *base = p.base[my_src];
-    const uint32_t W = (uint32_t)role_ctas * kGatherWarps;
-    const uint32_t gw = (uint32_t)my_idx * kGatherWarps + warp;
-    for (uint32_t e0 = gw * kRowsInFlight; e0 < cnt; e0 += W * kRowsInFlight)
-      copy_rows<kRowsInFlight>(base, p.out, R, b + e0, (int)min((uint32_t)kRowsInFlight, cnt - e0),
-                               lane);
+    stride_copy(p, b, cnt, base, (uint32_t)my_idx * kGatherWarps + warp,
+                (uint32_t)role_ctas * kGatherWarps, lane);
+  }
   }
   // local group: dedicated local CTAs start here; others pad once their group drains
   {

@@ -33,7 +33,7 @@ ugache_status resolve_params(const ugache_config *cfg, int device_sms, Params *p
   if (G < 1 || G > UGACHE_MAX_GPUS) return UGACHE_EINVAL;
   if (cfg->num_rows == 0 || cfg->num_rows >= (1ull << 32)) return UGACHE_EINVAL;
   if (cfg->row_bytes == 0 || (cfg->row_bytes % 16) != 0) return UGACHE_EINVAL;
-  if (cfg->reserved0 != 0 || cfg->flags != 0) return UGACHE_EINVAL;
+  if (cfg->reserved0 != 0 || (cfg->flags & ~UGACHE_FLAG_HOST_TIER) != 0) return UGACHE_EINVAL;
   if (cfg->policy < UGACHE_POLICY_UGACHE || cfg->policy > UGACHE_POLICY_PARTITION)
     return UGACHE_EINVAL;
   if (cfg->bw_local < 0 || cfg->bw_peer < 0 || cfg->bw_host < 0) return UGACHE_EINVAL;
@@ -281,6 +281,11 @@ ugache_status build_placement(const ugache_config *cfg, const uint32_t *order,
       const uint64_t owner = d % (uint64_t)G, slot = k + d / (uint64_t)G;
       loc[order[r]] = (owner << UGACHE_LOC_SRC_SHIFT) | slot;
     }
+    if (cfg->flags & UGACHE_FLAG_HOST_TIER) {  // host rows are tier slots: rank - band_end
+#pragma omp parallel for schedule(static)
+      for (int64_t r = (int64_t)be; r < (int64_t)N; ++r)
+        loc[order[r]] = host_tag | ((uint64_t)r - be);
+    }
   }
   uint64_t ns = k;
   if (be - k > (uint64_t)gpu) ns += (be - k - (uint64_t)gpu + (uint64_t)G - 1) / (uint64_t)G;
@@ -291,6 +296,25 @@ ugache_status build_placement(const ugache_config *cfg, const uint32_t *order,
   }
   if (n_slots) *n_slots = ns;
   return UGACHE_OK;
+}
+
+// tier[t] = table[order[be + t]] for t < N - be (parallel, first touch by the copying thread)
+template <typename OrderT>
+void fill_host_tier_impl(const uint8_t *table, uint32_t R, const OrderT *order, uint64_t be,
+                         uint64_t N, uint8_t *tier) {
+#pragma omp parallel for schedule(static)
+  for (int64_t t = 0; t < (int64_t)(N - be); ++t)
+    std::memcpy(tier + (uint64_t)t * R, table + (uint64_t)order[be + (uint64_t)t] * R, R);
+}
+
+void fill_host_tier(const uint8_t *table, uint32_t R, const uint64_t *order, uint64_t be,
+                    uint64_t N, uint8_t *tier) {
+  fill_host_tier_impl(table, R, order, be, N, tier);
+}
+
+void fill_host_tier(const uint8_t *table, uint32_t R, const uint32_t *order, uint64_t be,
+                    uint64_t N, uint8_t *tier) {
+  fill_host_tier_impl(table, R, order, be, N, tier);
 }
 
 }  // namespace ug
@@ -323,6 +347,27 @@ ugache_status ugache_build_placement(const ugache_config *cfg, const uint64_t *o
     ord[i] = (uint32_t)order[i];
   }
   return ug::build_placement(cfg, ord.data(), plan, gpu, loc, slot_keys, n_slots);
+}
+
+uint64_t ugache_host_tier_rows(const ugache_plan *plan, uint64_t num_rows) {
+  if (!plan || plan->band_end > num_rows) return 0;
+  return num_rows - plan->band_end;
+}
+
+ugache_status ugache_fill_host_tier(const ugache_config *cfg, const uint64_t *order,
+                                    const ugache_plan *plan, const void *host_table,
+                                    void *tier) {
+  if (!cfg || !order || !plan || !host_table) return UGACHE_EINVAL;
+  ug::Params p;
+  ugache_status st = ug::resolve_params(cfg, 0, &p);
+  if (st != UGACHE_OK) return st;
+  const uint64_t N = cfg->num_rows, be = plan->band_end;
+  if (be > N) return UGACHE_EINVAL;
+  if (be == N) return UGACHE_OK;
+  if (!tier) return UGACHE_EINVAL;
+  ug::fill_host_tier(static_cast<const uint8_t *>(host_table), cfg->row_bytes, order, be, N,
+                     static_cast<uint8_t *>(tier));
+  return UGACHE_OK;
 }
 
 }  // extern "C"

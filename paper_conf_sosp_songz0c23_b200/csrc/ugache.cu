@@ -4,6 +4,7 @@
 // ugache_extract -> K1 locate_bucket_kernel -> K2 factored_gather_kernel (kernels.cuh),
 // two launches on the caller's stream with no host synchronisation and no collective.
 #include <cuda_runtime.h>
+#include <sys/mman.h>
 
 #include <algorithm>
 #include <cstdio>
@@ -26,7 +27,11 @@ struct ugache_ctx {
   // host table (source G)
   const uint8_t *host_table = nullptr;
   const uint8_t *host_table_dev = nullptr;
-  bool registered = false;
+  std::vector<const void *> pinned;  // host ranges this ctx registered (refcounted globally)
+  // host tier (UGACHE_FLAG_HOST_TIER): rank-ordered copy of the host-resident rows
+  uint8_t *tier_owned = nullptr;
+  size_t tier_owned_bytes = 0;
+  const uint8_t *tier_dev = nullptr;
   // this GPU's cache slab and location table
   uint8_t *slab = nullptr;
   uint64_t slab_bytes = 0;
@@ -50,6 +55,10 @@ struct ugache_ctx {
   uint32_t *d_ranges = nullptr;  // 2 * kMaxRanges counters
   uint32_t range_shift = 0, n_ranges = 1;
   int host_sort = 1;
+  uint32_t host_sort_min = ugk::kHostSortMin;  // max(kHostSortMin, host 2 MB pages)
+  int host_dynamic = 1;  // size the host role from the host bucket when it is sparse
+  int warp_dedication = 0;            // UGACHE_OPT_DEDICATION
+  int wd_host_warps = 1, wd_peer_warps = 1;  // warp-granular dedication: warps per SM
   int host_warps = ugk::kHostWarps;  // env UGACHE_HOST_WARPS (A0 calibration knob)
   int stage_host_io = 0;             // env UGACHE_STAGE_HOST_IO=1: stage pinned host I/O too
   std::vector<int> smids;  // sorted %smid values of the device (one per SM)
@@ -135,41 +144,46 @@ bool is_pinned_host(const void *p) {
   return a.type == cudaMemoryTypeHost;
 }
 
-ugache_status register_host_table(ugache_ctx *ctx, const void *table, size_t bytes) {
-  std::lock_guard<std::mutex> lk(g_reg_mu);
-  auto it = g_reg_count.find(table);
-  if (it != g_reg_count.end()) {
-    it->second++;
-    ctx->registered = true;
-  } else if (!is_pinned_host(table)) {
-    cudaError_t e = cudaHostRegister(const_cast<void *>(table), bytes,
-                                     cudaHostRegisterMapped | cudaHostRegisterPortable |
-                                         cudaHostRegisterReadOnly);
-    if (e != cudaSuccess) {
-      (void)cudaGetLastError();
-      e = cudaHostRegister(const_cast<void *>(table), bytes,
-                           cudaHostRegisterMapped | cudaHostRegisterPortable);
+// Page-lock and map a host range (refcounted per address across contexts of the process)
+// and return its device address.  Already-pinned memory is used as is.
+ugache_status pin_host(ugache_ctx *ctx, const void *p, size_t bytes, const uint8_t **dev) {
+  {
+    std::lock_guard<std::mutex> lk(g_reg_mu);
+    auto it = g_reg_count.find(p);
+    if (it != g_reg_count.end()) {
+      it->second++;
+      ctx->pinned.push_back(p);
+    } else if (!is_pinned_host(p)) {
+      cudaError_t e = cudaHostRegister(const_cast<void *>(p), bytes,
+                                       cudaHostRegisterMapped | cudaHostRegisterPortable |
+                                           cudaHostRegisterReadOnly);
+      if (e != cudaSuccess) {
+        (void)cudaGetLastError();
+        e = cudaHostRegister(const_cast<void *>(p), bytes,
+                             cudaHostRegisterMapped | cudaHostRegisterPortable);
+      }
+      if (e != cudaSuccess) return cuda_fail(ctx, e, "cudaHostRegister");
+      g_reg_count[p] = 1;
+      ctx->pinned.push_back(p);
     }
-    if (e != cudaSuccess) return cuda_fail(ctx, e, "cudaHostRegister(host_table)");
-    g_reg_count[table] = 1;
-    ctx->registered = true;
   }
   void *dptr = nullptr;
-  UG_CUDA(ctx, cudaHostGetDevicePointer(&dptr, const_cast<void *>(table), 0));
-  ctx->host_table_dev = static_cast<const uint8_t *>(dptr);
+  UG_CUDA(ctx, cudaHostGetDevicePointer(&dptr, const_cast<void *>(p), 0));
+  *dev = static_cast<const uint8_t *>(dptr);
   return UGACHE_OK;
 }
 
-void unregister_host_table(ugache_ctx *ctx) {
-  if (!ctx->registered) return;
+void unpin_all(ugache_ctx *ctx) {
   std::lock_guard<std::mutex> lk(g_reg_mu);
-  auto it = g_reg_count.find(ctx->host_table);
-  if (it != g_reg_count.end() && --it->second == 0) {
-    cudaHostUnregister(const_cast<uint8_t *>(ctx->host_table));
-    (void)cudaGetLastError();
-    g_reg_count.erase(it);
+  for (const void *p : ctx->pinned) {
+    auto it = g_reg_count.find(p);
+    if (it != g_reg_count.end() && --it->second == 0) {
+      cudaHostUnregister(const_cast<void *>(p));
+      (void)cudaGetLastError();
+      g_reg_count.erase(it);
+    }
   }
-  ctx->registered = false;
+  ctx->pinned.clear();
 }
 
 ugache_status ensure_scratch(ugache_ctx *ctx, uint64_t n) {
@@ -205,53 +219,62 @@ ugache_status ensure_stage(ugache_ctx *ctx, void **buf, size_t *have, size_t nee
   return UGACHE_OK;
 }
 
-// Role table of the gather kernel: host SMs, then each peer's SMs, local
-// gets the rest.  SMs are handed out along a stride permutation of the sorted SM ids so
-// every role is spread over the whole chip (all GPCs / both dies) -- on the B200 box the
-// host source's zero-copy throughput scales with the number of GPCs issuing requests.
+// Core-dedication inputs of the gather kernel.  The roles themselves are
+// resolved on the device from the per-source counts: positions [0, H) of the SM order are
+// host SMs, then peer_sms positions per peer, then local.  The SM order is a stride
+// permutation of the sorted SM ids, so every role is spread over the whole chip (all GPCs,
+// both dies) -- on the B200 box the host source's zero-copy throughput scales with the
+// number of GPCs issuing requests.
 void build_roles(const ugache_ctx *ctx, ugk::GatherParams *gp, int *grid) {
   const int G = ctx->cfg.num_gpus, me = ctx->cfg.rank;
   const int S = (int)ctx->smids.size();
-  int nr = 0;
-  std::vector<int> want;
-  gp->role_src[nr] = G;  // host
-  want.push_back(ctx->host_sms);
-  ++nr;
-  for (int j = 0; j < G; ++j) {
-    if (j == me) continue;
-    gp->role_src[nr++] = j;
-    want.push_back(ctx->peer_sms);
-  }
-  int used = 0;
-  for (int w : want) used += w;
-  if (used < S) {
-    gp->role_src[nr++] = me;
-    want.push_back(S - used);
-  }
-  gp->n_roles = nr;
-  memset(gp->sm_role, nr - 1, sizeof(gp->sm_role));
-  memset(gp->sm_role_idx, 0, sizeof(gp->sm_role_idx));
+  gp->num_sms = S;
+  gp->host_sms = ctx->host_sms;
+  gp->peer_sms = G > 1 ? ctx->peer_sms : 0;
+  gp->n_peers = 0;
+  for (int j = 0; j < G; ++j)
+    if (j != me) gp->peer_src[gp->n_peers++] = j;
+  gp->host_sms_max = ctx->host_dynamic ? std::max(ctx->host_sms, S - gp->n_peers * gp->peer_sms)
+                                       : ctx->host_sms;
+  gp->host_sort_min = ctx->host_sort_min;
+  gp->warp_dedication = ctx->warp_dedication;
+  gp->peer_warps = ctx->wd_peer_warps;
+  gp->host_warps = ctx->warp_dedication ? ctx->wd_host_warps : ctx->host_warps;
+  memset(gp->sm_pos, S - 1, sizeof(gp->sm_pos));
   int stride = (int)(S * 0.6180339887) | 1;
   while (std::__gcd(stride, S) != 1) stride += 2;
-  int pos = 0;
-  for (int r = 0; r < nr; ++r) {
-    gp->role_count[r] = want[r];
-    for (int i = 0; i < want[r]; ++i, ++pos) {
-      const int sm = ctx->smids[(size_t)((int64_t)pos * stride % S)];
-      gp->sm_role[sm] = (uint8_t)r;
-      gp->sm_role_idx[sm] = (uint8_t)i;
-    }
-  }
+  for (int pos = 0; pos < S; ++pos)
+    gp->sm_pos[ctx->smids[(size_t)((int64_t)pos * stride % S)]] = (uint8_t)pos;
   *grid = S;
 }
 
 ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void *host_table,
-                          const std::vector<uint32_t> &order) {
+                          const std::vector<uint32_t> &order, const void *host_tier) {
   const uint64_t N = cfg->num_rows, R = cfg->row_bytes;
   const int G = cfg->num_gpus;
-  ugache_status st = register_host_table(ctx, host_table, (size_t)(N * R));
+  ugache_status st = pin_host(ctx, host_table, (size_t)(N * R), &ctx->host_table_dev);
   if (st != UGACHE_OK) return st;
   ctx->host_table = static_cast<const uint8_t *>(host_table);
+  const uint64_t tier_rows = N - ctx->plan.band_end;
+  if ((cfg->flags & UGACHE_FLAG_HOST_TIER) && tier_rows) {
+    const void *tier = host_tier;
+    if (!tier) {  // build this ctx's own rank-ordered host tier
+      ctx->tier_owned_bytes = (size_t)(tier_rows * R);
+      void *m = mmap(nullptr, ctx->tier_owned_bytes, PROT_READ | PROT_WRITE,
+                     MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+      if (m == MAP_FAILED) {
+        ctx->tier_owned_bytes = 0;
+        return fail(ctx, UGACHE_ENOMEM, "mmap of the host tier failed");
+      }
+      madvise(m, ctx->tier_owned_bytes, MADV_HUGEPAGE);
+      ctx->tier_owned = static_cast<uint8_t *>(m);
+      ug::fill_host_tier(static_cast<const uint8_t *>(host_table), (uint32_t)R, order.data(),
+                         ctx->plan.band_end, N, ctx->tier_owned);
+      tier = ctx->tier_owned;
+    }
+    st = pin_host(ctx, tier, (size_t)(tier_rows * R), &ctx->tier_dev);
+    if (st != UGACHE_OK) return st;
+  }
 
   // location table and slot list of this rank
   std::vector<uint64_t> loc;
@@ -283,11 +306,19 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   ctx->range_shift = 0;
   while (((N - 1) >> ctx->range_shift) + 1 > (uint64_t)ugk::kMaxRanges) ++ctx->range_shift;
   ctx->n_ranges = (uint32_t)(((N - 1) >> ctx->range_shift) + 1);
+  {  // ordering pays once host rows share translation pages: >= 1 key per 2 MB of host source
+    const uint64_t host_rows = ctx->tier_dev ? N - ctx->plan.band_end : N;
+    const uint64_t pages = (host_rows * R) >> 21;
+    ctx->host_sort_min = (uint32_t)std::min<uint64_t>(std::max<uint64_t>(ugk::kHostSortMin, pages),
+                                                      0xFFFFFFFFull);
+  }
+  if (const char *e = getenv("UGACHE_HOST_SORT_MIN")) ctx->host_sort_min = (uint32_t)atoll(e);
+  if (const char *e = getenv("UGACHE_HOST_DYNAMIC")) ctx->host_dynamic = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_HOST_WARPS")) ctx->host_warps = std::max(1, std::min(ugk::kGatherWarps, atoi(e)));
   for (int i = 0; i < 3; ++i) UG_CUDA(ctx, cudaEventCreate(&ctx->ev[i]));
   ctx->src_base[cfg->rank] = ctx->slab;
-  ctx->src_base[G] = ctx->host_table_dev;
+  ctx->src_base[G] = ctx->tier_dev ? ctx->tier_dev : ctx->host_table_dev;
   ctx->peers_ready = (G == 1);
   ctx->host_sms = ctx->plan.host_sms;
   ctx->peer_sms = ctx->plan.peer_sms;
@@ -349,7 +380,7 @@ const char *ugache_last_error_message(const ugache_ctx *ctx) {
 
 static ugache_status init_impl(ugache_ctx **out, const ugache_config *cfg, const void *host_table,
                                const float *hotness, const uint64_t *order_in,
-                               const ugache_plan *plan_in) {
+                               const ugache_plan *plan_in, const void *host_tier) {
   if (!out || !cfg || !host_table) return UGACHE_EINVAL;
   *out = nullptr;
   if (cfg->rank < 0 || cfg->rank >= cfg->num_gpus) return UGACHE_EINVAL;
@@ -390,7 +421,7 @@ static ugache_status init_impl(ugache_ctx **out, const ugache_config *cfg, const
     }
     if (st == UGACHE_OK && ctx->plan.num_sms > ctx->sm_count) st = UGACHE_EINVAL;
   }
-  if (st == UGACHE_OK) st = init_common(ctx, cfg, host_table, order);
+  if (st == UGACHE_OK) st = init_common(ctx, cfg, host_table, order, host_tier);
   if (st != UGACHE_OK) {
     ugache_destroy(ctx);
     return st;
@@ -401,14 +432,14 @@ static ugache_status init_impl(ugache_ctx **out, const ugache_config *cfg, const
 
 ugache_status ugache_init(ugache_ctx **ctx, const ugache_config *cfg, const void *host_table,
                           const float *hotness) {
-  return init_impl(ctx, cfg, host_table, hotness, nullptr, nullptr);
+  return init_impl(ctx, cfg, host_table, hotness, nullptr, nullptr, nullptr);
 }
 
 ugache_status ugache_init_with_plan(ugache_ctx **ctx, const ugache_config *cfg,
                                     const void *host_table, const uint64_t *order,
-                                    const ugache_plan *plan) {
+                                    const ugache_plan *plan, const void *host_tier) {
   if (!order || !plan) return UGACHE_EINVAL;
-  return init_impl(ctx, cfg, host_table, nullptr, order, plan);
+  return init_impl(ctx, cfg, host_table, nullptr, order, plan, host_tier);
 }
 
 ugache_status ugache_get_plan(const ugache_ctx *ctx, ugache_plan *plan) {
@@ -534,6 +565,19 @@ ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value) 
       if (value < 1 || value > ugk::kGatherWarps) return UGACHE_EINVAL;
       ctx->host_warps = (int)value;
       return UGACHE_OK;
+    case UGACHE_OPT_DEDICATION:
+      if (value != UGACHE_DEDICATE_SMS && value != UGACHE_DEDICATE_WARPS) return UGACHE_EINVAL;
+      ctx->warp_dedication = value == UGACHE_DEDICATE_WARPS;
+      return UGACHE_OK;
+    case UGACHE_OPT_WARP_HOST:
+    case UGACHE_OPT_WARP_PEER: {
+      const int hw = option == UGACHE_OPT_WARP_HOST ? (int)value : ctx->wd_host_warps;
+      const int pw = option == UGACHE_OPT_WARP_PEER ? (int)value : ctx->wd_peer_warps;
+      if (value < 1 || hw + (ctx->cfg.num_gpus - 1) * pw > ugk::kGatherWarps) return UGACHE_EINVAL;
+      ctx->wd_host_warps = hw;
+      ctx->wd_peer_warps = pw;
+      return UGACHE_OK;
+    }
   }
   return UGACHE_EINVAL;
 }
@@ -746,7 +790,8 @@ ugache_status ugache_destroy(ugache_ctx *ctx) {
     for (int i = 0; i < 3; ++i)
       if (ctx->ev[i]) cudaEventDestroy(ctx->ev[i]);
   }
-  unregister_host_table(ctx);
+  unpin_all(ctx);
+  if (ctx->tier_owned) munmap(ctx->tier_owned, ctx->tier_owned_bytes);
   (void)cudaGetLastError();
   delete ctx;
   return UGACHE_OK;

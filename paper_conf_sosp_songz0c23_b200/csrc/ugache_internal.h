@@ -35,5 +35,9 @@ ugache_status solve(const ugache_config *cfg, int device_sms, const float *hotne
 ugache_status build_placement(const ugache_config *cfg, const uint32_t *order,
                               const ugache_plan *plan, int gpu, uint64_t *loc,
                               uint64_t *slot_keys, uint64_t *n_slots);
+void fill_host_tier(const uint8_t *table, uint32_t R, const uint64_t *order, uint64_t be,
+                    uint64_t N, uint8_t *tier);
+void fill_host_tier(const uint8_t *table, uint32_t R, const uint32_t *order, uint64_t be,
+                    uint64_t N, uint8_t *tier);
 
 }  // namespace ug

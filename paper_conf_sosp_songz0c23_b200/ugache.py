@@ -44,12 +44,24 @@ def _stream_handle(stream) -> int:
 def make_config(num_rows: int, row_bytes: int, capacity_rows: int, num_gpus: int = 1,
                 rank: int = 0, device: int = 0, policy: str = "ugache", bw_local: float = 0.0,
                 bw_peer: float = 0.0, bw_host: float = 0.0, host_sms: int = 0,
-                peer_sms: int = 0, num_sms: int = 0) -> ugache_config:
+                peer_sms: int = 0, num_sms: int = 0, host_tier: bool = False) -> ugache_config:
     return ugache_config(num_rows=num_rows, row_bytes=row_bytes, reserved0=0,
                          capacity_rows=capacity_rows, num_gpus=num_gpus, rank=rank,
                          device=device, policy=_abi.POLICIES[policy] if isinstance(policy, str) else policy,
                          bw_local=bw_local, bw_peer=bw_peer, bw_host=bw_host,
-                         host_sms=host_sms, peer_sms=peer_sms, num_sms=num_sms, flags=0)
+                         host_sms=host_sms, peer_sms=peer_sms, num_sms=num_sms,
+                         flags=_abi.FLAG_HOST_TIER if host_tier else 0)
+
+
+def host_tier_rows(plan: ugache_plan, num_rows: int) -> int:
+    return int(lib().ugache_host_tier_rows(ctypes.byref(plan), num_rows))
+
+
+def fill_host_tier(cfg: ugache_config, order: np.ndarray, plan: ugache_plan, table, tier):
+    """Host-only: tier[t] = table[order[band_end + t]] (ugache_fill_host_tier)."""
+    order = np.ascontiguousarray(order, dtype=np.uint64)
+    check(lib().ugache_fill_host_tier(ctypes.byref(cfg), _ptr(order), ctypes.byref(plan),
+                                      _ptr(table), _ptr(tier)), "ugache_fill_host_tier")
 
 
 def solve(cfg: ugache_config, hotness: Optional[np.ndarray], want_order: bool = True):
@@ -80,15 +92,19 @@ class UGache:
     def __init__(self, table, num_rows: int, row_bytes: int, capacity_rows: int,
                  hotness: Optional[np.ndarray] = None, num_gpus: int = 1, rank: int = 0,
                  device: int = 0, policy: str = "ugache", plan: Optional[ugache_plan] = None,
-                 order: Optional[np.ndarray] = None, **model):
-        self._table = table  # keep the host buffer alive for the ctx's lifetime
+                 order: Optional[np.ndarray] = None, host_tier=False, **model):
+        """host_tier: False; True (the ctx builds its own rank-ordered host tier); or a
+        host buffer already filled by :func:`fill_host_tier` (shared by ranks)."""
+        self._table = table  # keep the host buffers alive for the ctx's lifetime
+        self._tier = host_tier if not isinstance(host_tier, bool) else None
         self.cfg = make_config(num_rows, row_bytes, capacity_rows, num_gpus, rank, device,
-                               policy, **model)
+                               policy, host_tier=host_tier is not False, **model)
         self.ctx = ctypes.c_void_p()
         if plan is not None and order is not None:
             order = np.ascontiguousarray(order, dtype=np.uint64)
             st = lib().ugache_init_with_plan(ctypes.byref(self.ctx), ctypes.byref(self.cfg),
-                                             _ptr(table), _ptr(order), ctypes.byref(plan))
+                                             _ptr(table), _ptr(order), ctypes.byref(plan),
+                                             _ptr(self._tier))
         else:
             h = None if hotness is None else np.ascontiguousarray(hotness, dtype=np.float32)
             st = lib().ugache_init(ctypes.byref(self.ctx), ctypes.byref(self.cfg), _ptr(table),
@@ -141,6 +157,15 @@ class UGache:
 
     def set_host_ordering(self, on: bool):
         self.set_option(_abi.OPT_HOST_ORDERING, int(on))
+
+    def set_dedication_mode(self, mode: str, host_warps: int = 0, peer_warps: int = 0):
+        """'sms' (whole SMs per source, the paper's) or 'warps' (warps per source on every SM)."""
+        self.set_option(_abi.OPT_DEDICATION,
+                        {"sms": _abi.DEDICATE_SMS, "warps": _abi.DEDICATE_WARPS}[mode])
+        if host_warps:
+            self.set_option(_abi.OPT_WARP_HOST, host_warps)
+        if peer_warps:
+            self.set_option(_abi.OPT_WARP_PEER, peer_warps)
 
     def set_stage_host_io(self, on: bool):
         self.set_option(_abi.OPT_STAGE_HOST_IO, int(on))

@@ -41,7 +41,7 @@ def test_struct_layouts_match_header():
 
 @pytest.mark.parametrize("field,value", [
     ("num_rows", 0), ("num_rows", 1 << 32), ("row_bytes", 0), ("row_bytes", 24),
-    ("num_gpus", 0), ("num_gpus", 17), ("policy", 3), ("flags", 1), ("reserved0", 2),
+    ("num_gpus", 0), ("num_gpus", 17), ("policy", 3), ("flags", 2), ("reserved0", 2),
     ("host_sms", 148), ("host_sms", -1), ("bw_host", -1.0)])
 def test_solve_rejects_bad_config(field, value):
     cfg = make_config(1000, 512, 100, num_gpus=2)
@@ -155,3 +155,36 @@ def test_solver_scale_pa_shaped():
     plan, order = solve(cfg, h)
     assert time.time() - t < 60
     assert np.all(np.diff(h[order.astype(np.int64)[:100000]]) <= 0)
+
+
+
+@pytest.mark.parametrize("N,C,G,alpha,kind", CASES[:6])
+def test_solver_host_tier_matches_oracle(N, C, G, alpha, kind):
+    h = _hot(N, alpha, kind)
+    cfg = make_config(N, 512, C, num_gpus=G, host_sms=8, host_tier=True)
+    plan, order = solve(cfg, h)
+    loc_ref, sk_ref = policy_placement(rank_order(h, N), N, C, G, int(plan.k), host_tier=True)
+    locs, sks = [], []
+    for g in range(G):
+        loc, sk = build_placement(cfg, order, plan, g)
+        assert np.array_equal(loc, loc_ref[g]) and np.array_equal(sk, sk_ref[g])
+        locs.append(loc)
+        sks.append(sk)
+    check_placement(np.stack(locs), sks, N, min(C, N),
+                    tier_keys=rank_order(h, N)[int(plan.band_end):])
+
+
+def test_fill_host_tier_matches_generator():
+    from paper_conf_sosp_songz0c23_b200 import fill_host_tier, host_tier_rows
+    N, R = 5000, 512
+    h = _hot(N, 1.2, "zipf")
+    cfg = make_config(N, R, 300, num_gpus=4, host_sms=8, host_tier=True)
+    plan, order = solve(cfg, h)
+    t = synth.make_table(N, R)
+    rows = host_tier_rows(plan, N)
+    assert rows == N - plan.band_end
+    tier = np.empty((rows, R), dtype=np.uint8)
+    fill_host_tier(cfg, order, plan, t, tier)
+    keys = order.astype(np.int64)[plan.band_end:]
+    assert np.array_equal(tier, synth.rows_for_keys(keys, N, R))
+    t.close()

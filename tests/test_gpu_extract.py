@@ -283,3 +283,60 @@ def test_pinned_host_io_zero_copy_and_staged(torch_cuda, staged):
         assert nbad == bad
     for c in group:
         c.close()
+
+
+@pytest.mark.parametrize("G", [1, 4])
+def test_host_tier_parity(torch_cuda, G):
+    """UGACHE_FLAG_HOST_TIER: host rows are read from the ctx's rank-ordered pinned copy."""
+    N, R = 300_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(11).permutation(N)]
+    t, group = make_group(torch_cuda, N, R, 3000, G, h, host_tier=True)
+    keys = np.random.default_rng(12).integers(-5, N + 5, 40_000)
+    for g, c in enumerate(group):
+        per = check_batch(torch_cuda, c, t, keys, N, R, G)
+        assert per[G] > 4096            # range-ordered host path on the tier
+        c.set_host_ordering(False)
+        check_batch(torch_cuda, c, t, keys[:999], N, R, G)
+    for c in group:
+        c.close()
+
+
+def test_shared_host_tier_buffer(torch_cuda):
+    """A caller-built tier (ugache_fill_host_tier) shared by every rank's ctx."""
+    from paper_conf_sosp_songz0c23_b200 import (UGache, connect_in_process, fill_host_tier,
+                                                host_tier_rows, make_config, solve)
+    wl = synth.get_workload("tiny")
+    N, R, G = wl.num_rows, wl.row_bytes, 2
+    t = table_for(N, R)
+    h = synth.hotness(wl)
+    cfg = make_config(N, R, wl.capacity_rows, num_gpus=G, host_tier=True)
+    plan, order = solve(cfg, h)
+    tier = np.empty((host_tier_rows(plan, N), R), dtype=np.uint8)
+    fill_host_tier(cfg, order, plan, t, tier)
+    group = [UGache(t, N, R, wl.capacity_rows, num_gpus=G, rank=g, plan=plan, order=order,
+                    host_tier=tier) for g in range(G)]
+    connect_in_process(group)
+    for c in group:
+        c.fill()
+    for g, c in enumerate(group):
+        check_batch(torch_cuda, c, t, synth.make_batch(wl, g, 2), N, R, G)
+    for c in group:
+        c.close()
+
+
+@pytest.mark.parametrize("G,hw,pw", [(1, 1, 1), (1, 5, 1), (4, 1, 1), (4, 3, 2), (8, 2, 2)])
+@pytest.mark.parametrize("big_host", [False, True])
+def test_warp_granular_dedication_parity(torch_cuda, G, hw, pw, big_host):
+    """UGACHE_DEDICATE_WARPS: host / peer warps on every SM, ordered or strided host reads."""
+    N, R = 300_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(13).permutation(N)]
+    C = 2000 if big_host else 60_000
+    t, group = make_group(torch_cuda, N, R, min(C, N // G), G, h)
+    keys = np.random.default_rng(14).integers(-3, N + 3, 30_000)
+    for g, c in enumerate(group):
+        c.set_dedication_mode("warps", host_warps=hw, peer_warps=pw)
+        per = check_batch(torch_cuda, c, t, keys, N, R, G)
+        if big_host:
+            assert per[G] > 4096
+    for c in group:
+        c.close()

@@ -219,3 +219,24 @@ def test_paper_policy_claims_model_level():
     loc_p, glob_p = hits(0, C_big)
     assert loc_u > 2 * loc_p
     assert glob_p - glob_u < 0.05
+
+
+def test_host_tier_worked_example():
+    """Host tier (R24) on the worked example: sweep k=1, C=2, G=2 gives
+    band_end = 1 + 2*(2-1) = 3, so ranks 3,4,5 (keys 3,4,5) sit in tier slots 0,1,2."""
+    N, G, C = 6, 2, 2
+    h = np.array([6, 5, 4, 3, 2, 1], dtype=np.float32)
+    order = rank_order(h, N)
+    loc, sk = policy_placement(order, N, C, G, 1, host_tier=True)
+    for g in range(G):
+        for key, slot in ((3, 0), (4, 1), (5, 2)):
+            s, r = dec(loc[g][key])
+            assert (int(s), int(r)) == (G, slot)
+    s, r = dec(loc[0][2])
+    assert (int(s), int(r)) == (1, 1)            # GPU entries unchanged
+    tier = order[3:]
+    check_placement(loc, sk, N, C, tier_keys=tier)
+    with pytest.raises(AssertionError):
+        check_placement(loc, sk, N, C, tier_keys=tier[::-1])
+    with pytest.raises(AssertionError):
+        check_placement(loc, sk, N, C)           # host rows are not keys any more
