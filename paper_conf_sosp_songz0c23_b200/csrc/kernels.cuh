@@ -95,6 +95,7 @@ struct GatherParams {
                                    // warp mode: host warps on every SM
   int32_t peer_warps;              // warp mode: warps per peer on every SM
   int32_t warp_dedication;         // 0 = SM-granular roles (paper), 1 = warp-granular roles
+  int32_t host_rows;               // rows per warp step on the unordered host path (1,2,4,8)
 };
 
 struct RandomParams {
@@ -373,12 +374,24 @@ __device__ __forceinline__ void host_role_sorted(const GatherParams &p, const ui
   host_copy_ordered<kRowsInFlight>(p, cnt, threadIdx.x & 31);
 }
 
-// Static warp striding of W warps (this one = gw) over a bucket of cnt rows of one source.
+// Static warp striding of W warps (this one = gw) over a bucket of cnt rows of one source,
+// U rows per warp step.
+template <int U>
+__device__ __forceinline__ void stride_copy_u(const GatherParams &p, const uint64_t *b, uint32_t cnt,
+                                              const uint8_t *base, uint32_t gw, uint32_t W, int lane) {
+  for (uint32_t e0 = gw * U; e0 < cnt; e0 += W * U)
+    copy_rows<U>(base, p.out, p.row_bytes, b + e0, (int)min((uint32_t)U, cnt - e0), lane);
+}
+
 __device__ __forceinline__ void stride_copy(const GatherParams &p, const uint64_t *b, uint32_t cnt,
-                                            const uint8_t *base, uint32_t gw, uint32_t W, int lane) {
-  for (uint32_t e0 = gw * kRowsInFlight; e0 < cnt; e0 += W * kRowsInFlight)
-    copy_rows<kRowsInFlight>(base, p.out, p.row_bytes, b + e0,
-                             (int)min((uint32_t)kRowsInFlight, cnt - e0), lane);
+                                            const uint8_t *base, uint32_t gw, uint32_t W, int lane,
+                                            int rows = kRowsInFlight) {
+  switch (rows) {
+    case 1: stride_copy_u<1>(p, b, cnt, base, gw, W, lane); break;
+    case 2: stride_copy_u<2>(p, b, cnt, base, gw, W, lane); break;
+    case 4: stride_copy_u<4>(p, b, cnt, base, gw, W, lane); break;
+    default: stride_copy_u<kRowsInFlight>(p, b, cnt, base, gw, W, lane); break;
+  }
 }
 
 // ---------------------------------------------------------------------------- K2
@@ -407,7 +420,8 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
     if (host_dense) host_order(p, bh, n_host, pos, S, s_dyn);
     if (warp < hw) {
       if (host_dense) host_copy_ordered<kRowsInFlight>(p, n_host, lane);
-      else stride_copy(p, bh, n_host, p.base[host_src], (uint32_t)(pos * hw + warp), (uint32_t)(S * hw), lane);
+      else stride_copy(p, bh, n_host, p.base[host_src], (uint32_t)(pos * hw + warp), (uint32_t)(S * hw), lane,
+                       p.host_rows);
     } else if (warp < hw + p.n_peers * pw) {
       const int j = p.peer_src[(warp - hw) / pw];
       stride_copy(p, p.buckets + (uint64_t)j * p.bucket_cap, p.ctrl->counts[j], p.base[j],
@@ -440,7 +454,8 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
     const uint64_t *b = p.buckets + (uint64_t)my_src * p.bucket_cap;
     const uint8_t *base = p.base[my_src];
     stride_copy(p, b, cnt, base, (uint32_t)my_idx * kGatherWarps + warp,
-                (uint32_t)role_ctas * kGatherWarps, lane);
+                (uint32_t)role_ctas * kGatherWarps, lane, my_src == host_src ? p.host_rows : kRowsInFlight);
+
   }
   }
   // local group: dedicated local CTAs start here; others pad once their group drains

@@ -59,6 +59,7 @@ struct ugache_ctx {
   int host_dynamic = 1;  // size the host role from the host bucket when it is sparse
   int warp_dedication = 0;            // UGACHE_OPT_DEDICATION
   int wd_host_warps = 1, wd_peer_warps = 1;  // warp-granular dedication: warps per SM
+  int host_rows = ugk::kRowsInFlight;        // env UGACHE_HOST_ROWS (1, 2, 4, 8)
   int host_warps = ugk::kHostWarps;  // env UGACHE_HOST_WARPS (A0 calibration knob)
   int stage_host_io = 0;             // env UGACHE_STAGE_HOST_IO=1: stage pinned host I/O too
   std::vector<int> smids;  // sorted %smid values of the device (one per SM)
@@ -238,6 +239,7 @@ void build_roles(const ugache_ctx *ctx, ugk::GatherParams *gp, int *grid) {
                                        : ctx->host_sms;
   gp->host_sort_min = ctx->host_sort_min;
   gp->warp_dedication = ctx->warp_dedication;
+  gp->host_rows = ctx->host_rows;
   gp->peer_warps = ctx->wd_peer_warps;
   gp->host_warps = ctx->warp_dedication ? ctx->wd_host_warps : ctx->host_warps;
   memset(gp->sm_pos, S - 1, sizeof(gp->sm_pos));
@@ -314,6 +316,7 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   }
   if (const char *e = getenv("UGACHE_HOST_SORT_MIN")) ctx->host_sort_min = (uint32_t)atoll(e);
   if (const char *e = getenv("UGACHE_HOST_DYNAMIC")) ctx->host_dynamic = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_HOST_ROWS")) ctx->host_rows = atoi(e);
   if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_HOST_WARPS")) ctx->host_warps = std::max(1, std::min(ugk::kGatherWarps, atoi(e)));
   for (int i = 0; i < 3; ++i) UG_CUDA(ctx, cudaEventCreate(&ctx->ev[i]));
