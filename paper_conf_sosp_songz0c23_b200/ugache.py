@@ -197,6 +197,9 @@ class UGache:
         if out is None:
             out = torch.empty((n, self.row_bytes), dtype=torch.uint8,
                               device=keys.device if hasattr(keys, "device") and keys.is_cuda else "cuda")
+        nbytes = out.nbytes if isinstance(out, np.ndarray) else out.numel() * out.element_size()
+        if nbytes < n * self.row_bytes:
+            raise ValueError(f"out holds {nbytes} bytes < n * row_bytes = {n * self.row_bytes}")
         check(lib().ugache_extract(self.ctx, _ptr(keys), kt, n, _ptr(out), _stream_handle(stream)),
               "ugache_extract", self.ctx)
         return out

@@ -340,3 +340,21 @@ def test_warp_granular_dedication_parity(torch_cuda, G, hw, pw, big_host):
             assert per[G] > 4096
     for c in group:
         c.close()
+
+
+def test_embedding_layer_module(torch_cuda):
+    """UGacheEmbedding: [B, T] keys -> [B, T, D] float32 rows, bitwise equal to
+    the oracle; no grad (read-only table)."""
+    from paper_conf_sosp_songz0c23_b200.layer import UGacheEmbedding
+    wl = synth.get_workload("tiny")
+    h = synth.hotness(wl)
+    t, (c,) = make_group(torch_cuda, wl.num_rows, 512, wl.capacity_rows, 1, h)
+    emb = UGacheEmbedding(c, 128, torch_cuda.float32)
+    keys_np = synth.make_batch(wl, 0, 7)[:4096].reshape(64, 64)
+    y = emb(torch_cuda.from_numpy(keys_np).cuda())
+    assert y.shape == (64, 64, 128) and y.dtype == torch_cuda.float32 and not y.requires_grad
+    ref, _ = oracle.gather(t.ptr, wl.num_rows, 512, keys_np.reshape(-1))
+    assert np.array_equal(y.view(torch_cuda.uint8).reshape(-1, 512).cpu().numpy(), ref)
+    with pytest.raises(ValueError):
+        UGacheEmbedding(c, 64, torch_cuda.float32)
+    c.close()
