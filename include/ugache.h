@@ -157,6 +157,17 @@ ugache_status ugache_init_with_plan(ugache_ctx **ctx, const ugache_config *cfg,
                                     const void *host_table, const uint64_t *order,
                                     const ugache_plan *plan, const void *host_tier);
 
+/* Same, with a placement computed elsewhere (e.g. the block-level MILP of section 6.3,
+ * P:1520-1566, which may replicate an entry on any subset of GPUs): loc = this GPU's
+ * location table (N entries, UGACHE_LOC_* encoding, host rows = keys), slot_keys = the keys
+ * of its slots 0..n_slots-1 (n_slots <= capacity_rows).  Checked: every key resolves to
+ * GPU j < G with row < capacity, or to the host with row == key; every key mapped to this
+ * GPU sits in the named slot.  UGACHE_FLAG_HOST_TIER is not supported here (EINVAL).  The
+ * plan reports policy -1, k = 0, band_end = N, z = 0. */
+ugache_status ugache_init_with_placement(ugache_ctx **ctx, const ugache_config *cfg,
+                                         const void *host_table, const uint64_t *loc,
+                                         const uint64_t *slot_keys, uint64_t n_slots);
+
 ugache_status ugache_get_plan(const ugache_ctx *ctx, ugache_plan *plan);
 
 /* Device address and size of this GPU's cache slab (for in-process peers / checks). */

@@ -167,7 +167,7 @@ def solve_sweep(h: np.ndarray, N: int, C: int, plat: Platform):
 
 # ----------------------------------------------------------------------------- checker
 def check_placement(loc: np.ndarray, slot_keys: List[np.ndarray], N: int, C: int,
-                    tier_keys: Optional[np.ndarray] = None):
+                    tier_keys: Optional[np.ndarray] = None, local_preference: bool = True):
     """Placement invariants (SURVEY.md section 8(c) checker items 1-4); raises AssertionError.
 
     1. resolution: LT_g[k] = (host, k) [or (host, t) with tier_keys[t] == k for a host
@@ -176,8 +176,9 @@ def check_placement(loc: np.ndarray, slot_keys: List[np.ndarray], N: int, C: int
        location in the format of <GPU_i, Offset>", P:946-952);
     2. capacity: n_slots_j <= C  (sum_e s^e_j <= Cap_j, P:1346-1353);
     3. storage covers access (s^e_j >= a^e_{i<-j}, P:1346) -- implied by 1;
-    4. local preference: an entry stored on g is read locally by g, and no GPU stores an
-       entry twice."""
+    4. local preference: an entry stored on g is read locally by g (the replicate/partition
+       family's arrangement; the section 6.2 MILP may choose otherwise, so callers checking
+       a MILP placement pass local_preference=False), and no GPU stores an entry twice."""
     G = loc.shape[0]
     for j in range(G):
         assert len(slot_keys[j]) <= C, f"GPU {j}: {len(slot_keys[j])} slots > capacity {C}"
@@ -200,9 +201,10 @@ def check_placement(loc: np.ndarray, slot_keys: List[np.ndarray], N: int, C: int
             sk = np.asarray(slot_keys[j], dtype=np.int64)
             assert np.all(row[m] < len(sk)), f"GPU {g}: slot beyond GPU {j}'s filled slots"
             assert np.all(sk[row[m]] == keys[m]), f"GPU {g}: GPU {j} slot holds another key"
-        own = np.asarray(slot_keys[g], dtype=np.int64)
-        assert np.all(src[own] == g), f"GPU {g}: locally stored entry not read locally"
-        assert np.all(row[own] == np.arange(len(own))), f"GPU {g}: local slot mismatch"
+        if local_preference:
+            own = np.asarray(slot_keys[g], dtype=np.int64)
+            assert np.all(src[own] == g), f"GPU {g}: locally stored entry not read locally"
+            assert np.all(row[own] == np.arange(len(own))), f"GPU {g}: local slot mismatch"
 
 
 def source_counts(loc_g: np.ndarray, keys: np.ndarray, N: int, G: int) -> Tuple[np.ndarray, int]:

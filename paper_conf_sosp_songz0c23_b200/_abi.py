@@ -67,7 +67,9 @@ SIGNATURES = {
     "ugache_init": (_ST, [ctypes.POINTER(_P), ctypes.POINTER(ugache_config), _P, _P]),
     "ugache_init_with_plan": (_ST, [ctypes.POINTER(_P), ctypes.POINTER(ugache_config), _P, _P,
                                     ctypes.POINTER(ugache_plan), _P]),
-    "ugache_host_tier_rows": (_c.c_uint64, [ctypes.POINTER(ugache_plan), _c.c_uint64]),
+    "ugache_init_with_placement": (_ST, [ctypes.POINTER(_P), ctypes.POINTER(ugache_config), _P, _P,
+                                         _P, _c.c_uint64]),
+    "ugache_host_tier_rows":(_c.c_uint64, [ctypes.POINTER(ugache_plan), _c.c_uint64]),
     "ugache_fill_host_tier": (_ST, [ctypes.POINTER(ugache_config), _P, ctypes.POINTER(ugache_plan),
                                     _P, _P]),
     "ugache_get_plan": (_ST, [_P, ctypes.POINTER(ugache_plan)]),

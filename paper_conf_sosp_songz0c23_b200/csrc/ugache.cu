@@ -250,8 +250,33 @@ void build_roles(const ugache_ctx *ctx, ugk::GatherParams *gp, int *grid) {
   *grid = S;
 }
 
+// Caller-provided placement (ugache_init_with_placement): checks that this GPU's table
+// resolves every key to a valid source / row and that its own slots hold the keys that map
+// to them (peer slots are the peers' business; the placement checker covers them).
+ugache_status check_given_placement(ugache_ctx *ctx, const ugache_config *cfg, const uint64_t *loc,
+                                    const uint64_t *slots, uint64_t n_slots) {
+  const uint64_t N = cfg->num_rows, C = cfg->capacity_rows;
+  const int G = cfg->num_gpus, me = cfg->rank;
+  if (n_slots > C || (n_slots && !slots)) return fail(ctx, UGACHE_EINVAL, "slot list exceeds capacity");
+  for (uint64_t s = 0; s < n_slots; ++s)
+    if (slots[s] >= N) return fail(ctx, UGACHE_EINVAL, "slot key out of range");
+  bool ok = true;
+#pragma omp parallel for reduction(&& : ok)
+  for (int64_t k = 0; k < (int64_t)N; ++k) {
+    const uint64_t src = loc[k] >> UGACHE_LOC_SRC_SHIFT, row = loc[k] & UGACHE_LOC_ROW_MASK;
+    bool good = src <= (uint64_t)G;
+    if (good && src == (uint64_t)G) good = row == (uint64_t)k;
+    if (good && src == (uint64_t)me) good = row < n_slots && slots[row] == (uint64_t)k;
+    if (good && src < (uint64_t)G) good = row < C;
+    ok = ok && good;
+  }
+  return ok ? UGACHE_OK : fail(ctx, UGACHE_EINVAL, "location table does not resolve every key");
+}
+
 ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void *host_table,
-                          const std::vector<uint32_t> &order, const void *host_tier) {
+                          const std::vector<uint32_t> &order, const void *host_tier,
+                          const uint64_t *given_loc = nullptr, const uint64_t *given_slots = nullptr,
+                          uint64_t given_n = 0) {
   const uint64_t N = cfg->num_rows, R = cfg->row_bytes;
   const int G = cfg->num_gpus;
   ugache_status st = pin_host(ctx, host_table, (size_t)(N * R), &ctx->host_table_dev);
@@ -287,9 +312,17 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   } catch (const std::bad_alloc &) {
     return fail(ctx, UGACHE_ENOMEM, "host allocation of the location table failed");
   }
-  st = ug::build_placement(cfg, order.data(), &ctx->plan, cfg->rank, loc.data(), slots.data(),
-                           &ctx->n_slots);
-  if (st != UGACHE_OK) return fail(ctx, st, "build_placement failed");
+  if (given_loc) {
+    st = check_given_placement(ctx, cfg, given_loc, given_slots, given_n);
+    if (st != UGACHE_OK) return st;
+    std::memcpy(loc.data(), given_loc, N * sizeof(uint64_t));
+    if (given_n) std::memcpy(slots.data(), given_slots, given_n * sizeof(uint64_t));
+    ctx->n_slots = given_n;
+  } else {
+    st = ug::build_placement(cfg, order.data(), &ctx->plan, cfg->rank, loc.data(), slots.data(),
+                             &ctx->n_slots);
+    if (st != UGACHE_OK) return fail(ctx, st, "build_placement failed");
+  }
 
   ctx->slab_bytes = std::max<uint64_t>(ctx->plan.capacity_rows, 1) * R;
   UG_CUDA(ctx, cudaMalloc(&ctx->slab, ctx->slab_bytes));
@@ -383,7 +416,9 @@ const char *ugache_last_error_message(const ugache_ctx *ctx) {
 
 static ugache_status init_impl(ugache_ctx **out, const ugache_config *cfg, const void *host_table,
                                const float *hotness, const uint64_t *order_in,
-                               const ugache_plan *plan_in, const void *host_tier) {
+                               const ugache_plan *plan_in, const void *host_tier,
+                               const uint64_t *given_loc = nullptr,
+                               const uint64_t *given_slots = nullptr, uint64_t given_n = 0) {
   if (!out || !cfg || !host_table) return UGACHE_EINVAL;
   *out = nullptr;
   if (cfg->rank < 0 || cfg->rank >= cfg->num_gpus) return UGACHE_EINVAL;
@@ -403,7 +438,22 @@ static ugache_status init_impl(ugache_ctx **out, const ugache_config *cfg, const
     if (e != cudaSuccess) st = cuda_fail(ctx, e, "cudaDeviceGetAttribute");
   }
   std::vector<uint32_t> order;
-  if (st == UGACHE_OK) {
+  if (st == UGACHE_OK && given_loc) {  // caller-provided placement: no solve
+    ug::Params p;
+    st = ug::resolve_params(cfg, ctx->sm_count, &p);
+    if (st == UGACHE_OK && (cfg->flags & UGACHE_FLAG_HOST_TIER)) st = UGACHE_EINVAL;
+    if (st == UGACHE_OK) {
+      ugache_plan &pl = ctx->plan;
+      std::memset(&pl, 0, sizeof(pl));
+      pl.policy = -1;
+      pl.num_gpus = cfg->num_gpus;
+      pl.capacity_rows = std::min<uint64_t>(cfg->capacity_rows, cfg->num_rows);
+      pl.band_end = cfg->num_rows;  // no host tier
+      pl.T_local = p.T_L, pl.T_peer = p.T_P, pl.T_host = p.T_H;
+      pl.R_local = p.R_L, pl.R_peer = p.R_P, pl.R_host = p.R_H;
+      pl.host_sms = p.host_sms, pl.peer_sms = p.peer_sms, pl.num_sms = p.S;
+    }
+  } else if (st == UGACHE_OK) {
     if (order_in && plan_in) {
       ug::Params p;
       st = ug::resolve_params(cfg, ctx->sm_count, &p);
@@ -424,7 +474,8 @@ static ugache_status init_impl(ugache_ctx **out, const ugache_config *cfg, const
     }
     if (st == UGACHE_OK && ctx->plan.num_sms > ctx->sm_count) st = UGACHE_EINVAL;
   }
-  if (st == UGACHE_OK) st = init_common(ctx, cfg, host_table, order, host_tier);
+  if (st == UGACHE_OK)
+    st = init_common(ctx, cfg, host_table, order, host_tier, given_loc, given_slots, given_n);
   if (st != UGACHE_OK) {
     ugache_destroy(ctx);
     return st;
@@ -443,6 +494,13 @@ ugache_status ugache_init_with_plan(ugache_ctx **ctx, const ugache_config *cfg,
                                     const ugache_plan *plan, const void *host_tier) {
   if (!order || !plan) return UGACHE_EINVAL;
   return init_impl(ctx, cfg, host_table, nullptr, order, plan, host_tier);
+}
+
+ugache_status ugache_init_with_placement(ugache_ctx **ctx, const ugache_config *cfg,
+                                         const void *host_table, const uint64_t *loc,
+                                         const uint64_t *slot_keys, uint64_t n_slots) {
+  if (!loc) return UGACHE_EINVAL;
+  return init_impl(ctx, cfg, host_table, nullptr, nullptr, nullptr, nullptr, loc, slot_keys, n_slots);
 }
 
 ugache_status ugache_get_plan(const ugache_ctx *ctx, ugache_plan *plan) {

@@ -92,15 +92,22 @@ class UGache:
     def __init__(self, table, num_rows: int, row_bytes: int, capacity_rows: int,
                  hotness: Optional[np.ndarray] = None, num_gpus: int = 1, rank: int = 0,
                  device: int = 0, policy: str = "ugache", plan: Optional[ugache_plan] = None,
-                 order: Optional[np.ndarray] = None, host_tier=False, **model):
+                 order: Optional[np.ndarray] = None, host_tier=False, placement=None, **model):
         """host_tier: False; True (the ctx builds its own rank-ordered host tier); or a
-        host buffer already filled by :func:`fill_host_tier` (shared by ranks)."""
+        host buffer already filled by :func:`fill_host_tier` (shared by ranks).
+        placement: optional (loc[N] uint64, slot_keys uint64) of this GPU computed elsewhere
+        (ugache_init_with_placement), e.g. by :mod:`.milp_solver`."""
         self._table = table  # keep the host buffers alive for the ctx's lifetime
         self._tier = host_tier if not isinstance(host_tier, bool) else None
         self.cfg = make_config(num_rows, row_bytes, capacity_rows, num_gpus, rank, device,
                                policy, host_tier=host_tier is not False, **model)
         self.ctx = ctypes.c_void_p()
-        if plan is not None and order is not None:
+        if placement is not None:
+            loc = np.ascontiguousarray(placement[0], dtype=np.uint64)
+            sk = np.ascontiguousarray(placement[1], dtype=np.uint64)
+            st = lib().ugache_init_with_placement(ctypes.byref(self.ctx), ctypes.byref(self.cfg),
+                                                  _ptr(table), _ptr(loc), _ptr(sk), len(sk))
+        elif plan is not None and order is not None:
             order = np.ascontiguousarray(order, dtype=np.uint64)
             st = lib().ugache_init_with_plan(ctypes.byref(self.ctx), ctypes.byref(self.cfg),
                                              _ptr(table), _ptr(order), ctypes.byref(plan),

@@ -358,3 +358,37 @@ def test_embedding_layer_module(torch_cuda):
     with pytest.raises(ValueError):
         UGacheEmbedding(c, 64, torch_cuda.float32)
     c.close()
+
+
+def test_block_milp_placement_parity(torch_cuda):
+    """Placement from the block-level MILP (section 6.3), which may replicate a block on any
+    subset of GPUs and read a stored block from a peer, through ugache_init_with_placement."""
+    from paper_conf_sosp_songz0c23_b200 import UGache, connect_in_process, make_config, solve
+    from paper_conf_sosp_songz0c23_b200.milp_solver import (make_blocks, placement_from_blocks,
+                                                            solve_blocks)
+    from oracle.placement import rank_order
+    N, R, G, C = 20_000, 512, 4, 900
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(21).permutation(N)]
+    cfg = make_config(N, R, C, num_gpus=G)
+    plan, order = solve(cfg, h)
+    ordr = order.astype(np.int64)
+    blocks = make_blocks(h[ordr], G)
+    s, a, z, _ = solve_blocks(h[ordr], blocks, C, G, (plan.T_local, plan.T_peer, plan.T_host),
+                              (plan.R_local, plan.R_peer, plan.R_host), time_limit=60)
+    locs, sks = placement_from_blocks(ordr, blocks, s, a, N, G)
+    t = table_for(N, R)
+    group = [UGache(t, N, R, C, num_gpus=G, rank=g, placement=(locs[g], sks[g])) for g in range(G)]
+    connect_in_process(group)
+    for c in group:
+        c.fill()
+    keys = np.random.default_rng(22).integers(0, N, 20_000)
+    for g, c in enumerate(group):
+        loc, sk = c.export_placement()
+        assert np.array_equal(loc, locs[g]) and np.array_equal(sk, sks[g])
+        check_batch(torch_cuda, c, t, keys, N, R, G)
+    bad = locs[0].copy()
+    bad[int(sks[0][0]) if len(sks[0]) else 0] = np.uint64(G) << np.uint64(56)  # host row != key
+    with pytest.raises(Exception):
+        UGache(t, N, R, C, num_gpus=G, rank=0, placement=(bad, sks[0]))
+    for c in group:
+        c.close()
