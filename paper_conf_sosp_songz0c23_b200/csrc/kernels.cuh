@@ -111,6 +111,7 @@ struct RandomParams {
 };
 
 struct FillParams {
+  const uint64_t *slot_idx;   // destination slot of entry i (nullptr: slot i)
   const uint64_t *slot_keys;
   const uint8_t *table;  // device-mapped host table
   uint8_t *slab;
@@ -552,9 +553,13 @@ __global__ void __launch_bounds__(256) fill_kernel(const FillParams p) {
   for (uint64_t s0 = warp * kRowsInFlight; s0 < p.n_slots; s0 += W * kRowsInFlight) {
     const int nvalid = (int)min((uint64_t)kRowsInFlight, p.n_slots - s0);
     const uint64_t key = lane < nvalid ? p.slot_keys[s0 + lane] : 0ull;
-    uint64_t ku[kRowsInFlight];
+    const uint64_t dst = lane < nvalid ? (p.slot_idx ? p.slot_idx[s0 + lane] : s0 + lane) : 0ull;
+    uint64_t ku[kRowsInFlight], du[kRowsInFlight];
 #pragma unroll
-    for (int u = 0; u < kRowsInFlight; ++u) ku[u] = __shfl_sync(kFullMask, key, u);
+    for (int u = 0; u < kRowsInFlight; ++u) {
+      ku[u] = __shfl_sync(kFullMask, key, u);
+      du[u] = __shfl_sync(kFullMask, dst, u);
+    }
     for (uint32_t j = lane; j < V; j += 32) {
       uint4 v[kRowsInFlight];
 #pragma unroll
@@ -563,8 +568,21 @@ __global__ void __launch_bounds__(256) fill_kernel(const FillParams p) {
 #pragma unroll
       for (int u = 0; u < kRowsInFlight; ++u)
         if (u < nvalid)
-          *reinterpret_cast<uint4 *>(p.slab + (s0 + u) * p.row_bytes + (uint64_t)j * 16u) = v[u];
+          *reinterpret_cast<uint4 *>(p.slab + du[u] * p.row_bytes + (uint64_t)j * 16u) = v[u];
     }
+  }
+}
+
+// ---------------------------------------------------------------------------- refresh
+// Cache refresh, step 1: every key whose location changes is first pointed at
+// the host (which holds every entry), so no reader can reach a slot whose content is about
+// to be rewritten; unchanged locations stay.
+__global__ void __launch_bounds__(256) refresh_evict_kernel(uint64_t *loc, const uint64_t *loc_new,
+                                                            uint64_t N, uint64_t host_tag) {
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < N;
+       k += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t a = loc[k];
+    if (a != loc_new[k]) loc[k] = host_tag | k;
   }
 }
 

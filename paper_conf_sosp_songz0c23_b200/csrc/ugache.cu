@@ -37,7 +37,14 @@ struct ugache_ctx {
   uint64_t slab_bytes = 0;
   uint64_t n_slots = 0;
   uint64_t *d_slot_keys = nullptr;
+  uint64_t slot_keys_cap = 0;
+  std::vector<uint64_t> h_slot_keys;  // host copy of the slot list (refresh diffs)
   uint64_t *d_loc = nullptr;
+  // cache refresh: 0 idle, 1 evicted (LT transitional), 2 content written
+  int refresh_state = 0;
+  uint64_t *d_loc_new = nullptr;
+  std::vector<uint64_t> new_slot_keys;
+  uint64_t refresh_changed = 0;
   // sources
   const uint8_t *src_base[ug::kMaxSrc] = {};
   void *ipc_mapped[UGACHE_MAX_GPUS] = {};
@@ -332,7 +339,9 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
     UG_CUDA(ctx, cudaMalloc(&ctx->d_slot_keys, ctx->n_slots * sizeof(uint64_t)));
     UG_CUDA(ctx, cudaMemcpy(ctx->d_slot_keys, slots.data(), ctx->n_slots * sizeof(uint64_t),
                             cudaMemcpyHostToDevice));
+    ctx->slot_keys_cap = ctx->n_slots;
   }
+  ctx->h_slot_keys.assign(slots.begin(), slots.begin() + (ptrdiff_t)ctx->n_slots);
   UG_CUDA(ctx, cudaMalloc(&ctx->d_ctrl, sizeof(ugk::Ctrl)));
   UG_CUDA(ctx, cudaMemset(ctx->d_ctrl, 0, sizeof(ugk::Ctrl)));
   UG_CUDA(ctx, cudaMalloc(&ctx->d_ranges, 2 * ugk::kMaxRanges * sizeof(uint32_t)));
@@ -585,6 +594,7 @@ ugache_status ugache_fill(ugache_ctx *ctx, void *stream) {
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   if (ctx->n_slots) {
     ugk::FillParams fp;
+    fp.slot_idx = nullptr;
     fp.slot_keys = ctx->d_slot_keys;
     fp.table = ctx->host_table_dev;
     fp.slab = ctx->slab;
@@ -595,6 +605,102 @@ ugache_status ugache_fill(ugache_ctx *ctx, void *stream) {
     UG_CUDA(ctx, cudaGetLastError());
   }
   ctx->filled = true;
+  return UGACHE_OK;
+}
+
+// ---- cache refresh (section 7.2) -------------------------------------------
+ugache_status ugache_refresh_begin(ugache_ctx *ctx, const uint64_t *new_loc,
+                                   const uint64_t *new_slot_keys, uint64_t n_new_slots,
+                                   void *stream) {
+  if (!ctx || !new_loc) return UGACHE_EINVAL;
+  if (ctx->refresh_state != 0) return fail(ctx, UGACHE_ESTATE, "refresh already in progress");
+  if (!ctx->filled) return fail(ctx, UGACHE_ESTATE, "refresh before fill");
+  if (ctx->tier_dev) return fail(ctx, UGACHE_EINVAL, "refresh of a host-tier ctx is not supported");
+  ugache_status st = check_given_placement(ctx, &ctx->cfg, new_loc, new_slot_keys, n_new_slots);
+  if (st != UGACHE_OK) return st;
+  st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  const uint64_t N = ctx->cfg.num_rows;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  UG_CUDA(ctx, cudaStreamSynchronize(s));
+  if (!ctx->d_loc_new) UG_CUDA(ctx, cudaMalloc(&ctx->d_loc_new, N * sizeof(uint64_t)));
+  UG_CUDA(ctx, cudaMemcpy(ctx->d_loc_new, new_loc, N * sizeof(uint64_t), cudaMemcpyHostToDevice));
+  ctx->new_slot_keys.assign(new_slot_keys, new_slot_keys + n_new_slots);
+  const uint64_t host_tag = (uint64_t)ctx->cfg.num_gpus << UGACHE_LOC_SRC_SHIFT;
+  ugk::refresh_evict_kernel<<<ctx->sm_count * 8, 256, 0, s>>>(ctx->d_loc, ctx->d_loc_new, N, host_tag);
+  UG_CUDA(ctx, cudaGetLastError());
+  ctx->refresh_state = 1;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_refresh_content(ugache_ctx *ctx, int32_t max_sms, void *stream) {
+  if (!ctx || max_sms < 0) return UGACHE_EINVAL;
+  if (ctx->refresh_state != 1) return fail(ctx, UGACHE_ESTATE, "refresh_content before refresh_begin");
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  std::vector<uint64_t> idx, keys;
+  for (uint64_t i = 0; i < ctx->new_slot_keys.size(); ++i)
+    if (i >= ctx->h_slot_keys.size() || ctx->h_slot_keys[i] != ctx->new_slot_keys[i]) {
+      idx.push_back(i);
+      keys.push_back(ctx->new_slot_keys[i]);
+    }
+  ctx->refresh_changed = idx.size();
+  if (!idx.empty()) {
+    uint64_t *d = nullptr;
+    UG_CUDA(ctx, cudaMalloc(&d, 2 * idx.size() * sizeof(uint64_t)));
+    cudaError_t e = cudaMemcpy(d, idx.data(), idx.size() * 8, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = cudaMemcpy(d + idx.size(), keys.data(), keys.size() * 8, cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+      cudaFree(d);
+      return cuda_fail(ctx, e, "refresh staging");
+    }
+    ugk::FillParams fp;
+    fp.slot_idx = d;
+    fp.slot_keys = d + idx.size();
+    fp.table = ctx->host_table_dev;
+    fp.slab = ctx->slab;
+    fp.n_slots = idx.size();
+    fp.row_bytes = ctx->cfg.row_bytes;
+    // throttle: the refresh touches at most max_sms SMs' worth of CTAs
+    const int sms = max_sms ? std::min(max_sms, ctx->sm_count) : ctx->sm_count;
+    ugk::fill_kernel<<<sms * 8, 256, 0, s>>>(fp);
+    e = cudaGetLastError();
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    cudaFree(d);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "refresh fill");
+  }
+  ctx->refresh_state = 2;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_refresh_commit(ugache_ctx *ctx, void *stream) {
+  if (!ctx) return UGACHE_EINVAL;
+  if (ctx->refresh_state != 2) return fail(ctx, UGACHE_ESTATE, "refresh_commit before refresh_content");
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const uint64_t N = ctx->cfg.num_rows;
+  UG_CUDA(ctx, cudaMemcpyAsync(ctx->d_loc, ctx->d_loc_new, N * sizeof(uint64_t), cudaMemcpyDeviceToDevice, s));
+  const uint64_t ns = ctx->new_slot_keys.size();
+  if (ns > ctx->slot_keys_cap) {
+    UG_CUDA(ctx, cudaStreamSynchronize(s));
+    cudaFree(ctx->d_slot_keys);
+    ctx->d_slot_keys = nullptr;
+    UG_CUDA(ctx, cudaMalloc(&ctx->d_slot_keys, ns * sizeof(uint64_t)));
+    ctx->slot_keys_cap = ns;
+  }
+  if (ns)
+    UG_CUDA(ctx, cudaMemcpyAsync(ctx->d_slot_keys, ctx->new_slot_keys.data(), ns * sizeof(uint64_t),
+                                 cudaMemcpyHostToDevice, s));
+  UG_CUDA(ctx, cudaStreamSynchronize(s));
+  ctx->h_slot_keys.swap(ctx->new_slot_keys);
+  ctx->new_slot_keys.clear();
+  ctx->n_slots = ns;
+  cudaFree(ctx->d_loc_new);
+  ctx->d_loc_new = nullptr;
+  ctx->plan.policy = -1;  // the placement no longer comes from this ctx's solve
+  ctx->refresh_state = 0;
   return UGACHE_OK;
 }
 
@@ -848,6 +954,7 @@ ugache_status ugache_destroy(ugache_ctx *ctx) {
     cudaFree(ctx->d_out_stage);
     cudaFree(ctx->d_host_sorted);
     cudaFree(ctx->d_ranges);
+    cudaFree(ctx->d_loc_new);
     for (int i = 0; i < 3; ++i)
       if (ctx->ev[i]) cudaEventDestroy(ctx->ev[i]);
   }

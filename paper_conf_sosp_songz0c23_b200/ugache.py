@@ -152,6 +152,21 @@ class UGache:
     def fill(self, stream=None):
         check(lib().ugache_fill(self.ctx, _stream_handle(stream)), "ugache_fill", self.ctx)
 
+    # -- cache refresh (ugache_refresh_*) ------------------------------------
+    def refresh_begin(self, loc: np.ndarray, slot_keys: np.ndarray, stream=None):
+        loc = np.ascontiguousarray(loc, dtype=np.uint64)
+        sk = np.ascontiguousarray(slot_keys, dtype=np.uint64)
+        check(lib().ugache_refresh_begin(self.ctx, _ptr(loc), _ptr(sk), len(sk), _stream_handle(stream)),
+              "ugache_refresh_begin", self.ctx)
+
+    def refresh_content(self, max_sms: int = 0, stream=None):
+        check(lib().ugache_refresh_content(self.ctx, max_sms, _stream_handle(stream)),
+              "ugache_refresh_content", self.ctx)
+
+    def refresh_commit(self, stream=None):
+        check(lib().ugache_refresh_commit(self.ctx, _stream_handle(stream)), "ugache_refresh_commit",
+              self.ctx)
+
     def set_dedication(self, host_sms: int = 0, peer_sms: int = 0):
         check(lib().ugache_set_dedication(self.ctx, host_sms, peer_sms), "ugache_set_dedication", self.ctx)
 

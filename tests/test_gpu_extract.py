@@ -392,3 +392,68 @@ def test_block_milp_placement_parity(torch_cuda):
         UGache(t, N, R, C, num_gpus=G, rank=0, placement=(bad, sks[0]))
     for c in group:
         c.close()
+
+
+def test_cache_refresh_protocol(torch_cuda):
+    """Section 7.2 refresh on G = 3 fake peers: hotness shifts (a new Zipf permutation), the
+    Refresher re-solves, and extraction stays bit-exact after every step (transitional
+    table -> rewritten content -> new table); the committed placement equals the new one
+    and passes the checker; the modeled time of the old placement under the new hotness is
+    worse than the new optimum."""
+    from paper_conf_sosp_songz0c23_b200 import UGache, connect_in_process
+    from paper_conf_sosp_songz0c23_b200.refresh import (HotnessSampler, modeled_time,
+                                                        plan_placements, refresh_group,
+                                                        should_refresh)
+    N, R, G, C = 100_000, 512, 3, 6000
+    p = (synth.zipf_pmf(N, 1.2) * 8192).astype(np.float32)
+    h1 = p[np.random.default_rng(1).permutation(N)]
+    h2 = p[np.random.default_rng(2).permutation(N)]
+    kw = dict(num_rows=N, row_bytes=R, capacity_rows=C)
+    plan1, pl1 = plan_placements(kw, h1, G)
+    t = table_for(N, R)
+    group = [UGache(t, N, R, C, num_gpus=G, rank=g, placement=pl1[g]) for g in range(G)]
+    connect_in_process(group)
+    for c in group:
+        c.fill()
+    # foreground sampling under the new distribution
+    rng = np.random.default_rng(3)
+    cdf = np.cumsum(h2.astype(np.float64)) / h2.sum()
+    sampler = HotnessSampler(N)
+    batches = [np.searchsorted(cdf, rng.random(8192)).astype(np.int64) for _ in range(8)]
+    for b in batches:
+        sampler.record(b)
+    plan2, pl2 = plan_placements(kw, sampler.hotness(), G)
+    assert should_refresh([l for l, _ in pl1], h2, plan2)
+    assert modeled_time([l for l, _ in pl2], h2, plan2) < modeled_time([l for l, _ in pl1], h2, plan2)
+
+    def foreground():
+        for g, c in enumerate(group):
+            check_batch(torch_cuda, c, t, batches[g], N, R, G)
+
+    foreground()
+    for c, (loc, sk) in zip(group, pl2):
+        c.refresh_begin(loc, sk)
+    foreground()                                  # transitional tables
+    with pytest.raises(Exception):
+        group[0].refresh_commit()                 # content step missing -> ESTATE
+    for c in group:
+        c.refresh_content(max_sms=4)
+    foreground()                                  # new content, transitional tables
+    for c in group:
+        c.refresh_commit()
+    foreground()                                  # new placement
+    locs, sks = [], []
+    for g, c in enumerate(group):
+        loc, sk = c.export_placement()
+        assert np.array_equal(loc, pl2[g][0]) and np.array_equal(sk, pl2[g][1])
+        locs.append(loc)
+        sks.append(sk)
+        if len(sk):
+            idx = np.linspace(0, len(sk) - 1, 301).astype(np.int64)
+            assert np.array_equal(c.read_slab(0, len(sk))[idx], t.array[sk[idx].astype(np.int64)])
+    check_placement(np.stack(locs), sks, N, C)
+    # refresh back with the group helper
+    refresh_group(group, pl1, max_sms=8, foreground=foreground)
+    foreground()
+    for c in group:
+        c.close()
