@@ -56,10 +56,14 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--no-verify", action="store_true")
-    ap.add_argument("--extra", action="store_true", help="also time the random-dispatch ablation")
     ap.add_argument("--no-clocks", action="store_true", help="do not sample nvidia-smi (diagnostics only)")
-    ap.add_argument("--host-tier", action="store_true",
-                    help="read host rows from a hotness-ordered pinned copy (UGACHE_FLAG_HOST_TIER)")
+    ap.add_argument("--host-tier", dest="host_tier", action="store_true", default=True,
+                    help="read host rows from a hotness-ordered pinned copy (UGACHE_FLAG_HOST_TIER, "
+                         "default)")
+    ap.add_argument("--no-host-tier", dest="host_tier", action="store_false")
+    ap.add_argument("--extra", dest="extra", action="store_true", default=True,
+                    help="also time the random-dispatch (unfactored) ablation (default)")
+    ap.add_argument("--no-extra", dest="extra", action="store_false")
     return ap.parse_args()
 
 
