@@ -447,13 +447,23 @@ def main():
     step_hbm = (n * kb + n * 32 + n * 8 + n * 8) + gather_hbm_bytes
     t_roof = max(step_hbm / (hbm * 1e9), t_pcie, t_nvl)
     ms_per_step = statistics.mean(step_ms)
+    traffic = traffic_pcie = traffic_src = None
+    try:  # per-launch DRAM traffic of K2 from the committed ncu capture of this workload
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            rec = json.load(f)[wl.name]["factored_gather_kernel"]
+        traffic, traffic_pcie, traffic_src = rec["dram_bytes"], rec.get("pcie_read_bytes"), rec["source"]
+    except Exception:
+        pass
     line = {
         "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": ws, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
         "config": config_dict(args, wl, ws),
         "roofline": {"bound": bound, "achieved": achieved, "peak": peak, "unit": unit,
-                     "frac": achieved / peak if peak else None, "traffic": None,
+                     "frac": achieved / peak if peak else None, "traffic": traffic,
+                     "traffic_pcie_read": traffic_pcie, "traffic_source": traffic_src,
+                     "algorithmic_bytes": {"hbm": gather_hbm_bytes, "pcie": gather_pcie_bytes,
+                                           "nvlink": n_peer * R},
                      "kernel": "factored_gather_kernel", "peak_source": psrc,
                      "kernel_ms": statistics.mean(gat_ms)},
         "source_mix_roofline": {"t_roof_us": t_roof * 1e6, "t_step_us": ms_per_step * 1e3,
