@@ -244,14 +244,19 @@ ugache_status ugache_set_mode(ugache_ctx *ctx, int32_t mode);
  *    on every SM, UGACHE_OPT_WARP_HOST warps serve the host and UGACHE_OPT_WARP_PEER warps
  *    serve each peer, the others start on local rows.
  *  UGACHE_OPT_WARP_HOST / UGACHE_OPT_WARP_PEER (default 1 / 1): warps per SM in
- *    UGACHE_DEDICATE_WARPS mode; host + (G-1) * peer <= 16. */
+ *    UGACHE_DEDICATE_WARPS mode; host + (G-1) * peer <= 16.
+ *  UGACHE_OPT_HOST_WALK (default 1): when the host bucket is sparse (fewer keys than 2 MB
+ *    pages of host source), every SM not dedicated to a peer first walks the batch's keys in
+ *    input order and copies the host rows it meets (paced, input-ordered host requests),
+ *    then pads local work; 0 = copy the sparse host bucket with dedicated SMs. */
 typedef enum {
   UGACHE_OPT_HOST_ORDERING = 0,
   UGACHE_OPT_STAGE_HOST_IO = 1,
   UGACHE_OPT_HOST_WARPS = 2,
   UGACHE_OPT_DEDICATION = 3,
   UGACHE_OPT_WARP_HOST = 4,
-  UGACHE_OPT_WARP_PEER = 5
+  UGACHE_OPT_WARP_PEER = 5,
+  UGACHE_OPT_HOST_WALK = 6
 } ugache_option;
 typedef enum { UGACHE_DEDICATE_SMS = 0, UGACHE_DEDICATE_WARPS = 1 } ugache_dedication;
 ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value);

@@ -96,6 +96,13 @@ struct GatherParams {
   int32_t peer_warps;              // warp mode: warps per peer on every SM
   int32_t warp_dedication;         // 0 = SM-granular roles (paper), 1 = warp-granular roles
   int32_t host_rows;               // rows per warp step on the unordered host path (1,2,4,8)
+  // sparse host bucket: input-order walk over the batch (host_walk)
+  const void *keys;                // the batch's keys (device)
+  const uint64_t *loc;             // this GPU's location table
+  uint64_t num_rows;
+  uint32_t n_keys;
+  int32_t keys_u32;                // key type: 0 = int64, 1 = uint32
+  int32_t host_walk;               // 1 = sparse host buckets use the input-order walk
 };
 
 struct RandomParams {
@@ -433,8 +440,11 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
   // (throughput-bound); otherwise enough SMs to put the whole bucket in flight in about one
   // round (latency-bound), capped so every peer keeps its dedicated SMs.  Every CTA derives
   // the same split from the same counts.
+  const bool host_walk = p.host_walk && !host_dense && n_host > 0;
   int H = p.host_sms;
-  if (!host_dense)
+  if (host_walk)
+    H = p.host_sms_max;  // every SM not dedicated to a peer walks the batch for host rows
+  else if (!host_dense)
     H = max(H, min(p.host_sms_max, (int)((n_host + kRowsPerSmRound - 1) / kRowsPerSmRound)));
   int my_src, my_idx, role_ctas;
   if (pos < H) {
@@ -446,7 +456,34 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
     my_src = p.local_src, my_idx = 0, role_ctas = 0;
   }
 
-  if (my_src == host_src && host_dense) {
+  if (my_src == host_src && host_walk) {
+    // Sparse host bucket: the host SMs walk the batch's keys in input order (re-reading
+    // their location entries) and copy the host rows they meet.  Measured on the B200 box,
+    // sparse cold host rows are read ~1.6x faster in this paced input order than from the
+    // dense host bucket, whose rows would all be requested at once.
+    __shared__ uint64_t s_ent[kGatherWarps][kRowsInFlight];
+    const uint32_t W = (uint32_t)role_ctas * kGatherWarps;
+    for (uint32_t e0 = ((uint32_t)my_idx * kGatherWarps + warp) * kRowsInFlight; e0 < p.n_keys;
+         e0 += W * kRowsInFlight) {
+      const int nv = (int)min((uint32_t)kRowsInFlight, p.n_keys - e0);
+      uint64_t ent = ~0ull;
+      if (lane < nv) {
+        const uint64_t i = e0 + lane;
+        const int64_t k = p.keys_u32 ? (int64_t)static_cast<const uint32_t *>(p.keys)[i]
+                                     : static_cast<const int64_t *>(p.keys)[i];
+        if (k >= 0 && (uint64_t)k < p.num_rows) {
+          const uint64_t l = ld_nc_u64(p.loc + k);
+          if ((int)(l >> UGACHE_LOC_SRC_SHIFT) == host_src)
+            ent = ((l & UGACHE_LOC_ROW_MASK) << 32) | i;
+        }
+      }
+      const uint32_t m = __ballot_sync(kFullMask, ent != ~0ull);
+      if (ent != ~0ull) s_ent[warp][__popc(m & lanemask_lt())] = ent;  // compact to lanes 0..
+      __syncwarp();
+      if (m) copy_rows<kRowsInFlight>(p.base[host_src], p.out, R, s_ent[warp], __popc(m), lane);
+      __syncwarp();
+    }
+  } else if (my_src == host_src && host_dense) {
     host_role_sorted(p, p.buckets + (uint64_t)host_src * p.bucket_cap, n_host, my_idx, role_ctas,
                      s_dyn);
   } else if (my_src != p.local_src) {

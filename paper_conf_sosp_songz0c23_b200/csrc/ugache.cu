@@ -67,6 +67,7 @@ struct ugache_ctx {
   int warp_dedication = 0;            // UGACHE_OPT_DEDICATION
   int wd_host_warps = 1, wd_peer_warps = 1;  // warp-granular dedication: warps per SM
   int host_rows = ugk::kRowsInFlight;        // env UGACHE_HOST_ROWS (1, 2, 4, 8)
+  int host_walk = 1;                         // UGACHE_OPT_HOST_WALK
   int host_warps = ugk::kHostWarps;  // env UGACHE_HOST_WARPS (A0 calibration knob)
   int stage_host_io = 0;             // env UGACHE_STAGE_HOST_IO=1: stage pinned host I/O too
   std::vector<int> smids;  // sorted %smid values of the device (one per SM)
@@ -732,6 +733,7 @@ ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value) 
       if (value < 1 || value > ugk::kGatherWarps) return UGACHE_EINVAL;
       ctx->host_warps = (int)value;
       return UGACHE_OK;
+    case UGACHE_OPT_HOST_WALK: ctx->host_walk = value != 0; return UGACHE_OK;
     case UGACHE_OPT_DEDICATION:
       if (value != UGACHE_DEDICATE_SMS && value != UGACHE_DEDICATE_WARPS) return UGACHE_EINVAL;
       ctx->warp_dedication = value == UGACHE_DEDICATE_WARPS;
@@ -851,6 +853,12 @@ ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type
     gp.range_shift = ctx->range_shift;
     gp.n_ranges = ctx->n_ranges;
     gp.host_sort = ctx->host_sort;
+    gp.keys = dkeys;
+    gp.loc = ctx->d_loc;
+    gp.num_rows = ctx->cfg.num_rows;
+    gp.n_keys = (uint32_t)n;
+    gp.keys_u32 = key_type == UGACHE_KEY_U32;
+    gp.host_walk = ctx->host_walk;
     gp.host_warps = ctx->host_warps;
     int grid = 0;
     build_roles(ctx, &gp, &grid);

@@ -189,6 +189,9 @@ class UGache:
         if peer_warps:
             self.set_option(_abi.OPT_WARP_PEER, peer_warps)
 
+    def set_host_walk(self, on: bool):
+        self.set_option(_abi.OPT_HOST_WALK, int(on))
+
     def set_stage_host_io(self, on: bool):
         self.set_option(_abi.OPT_STAGE_HOST_IO, int(on))
 

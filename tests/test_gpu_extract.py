@@ -457,3 +457,24 @@ def test_cache_refresh_protocol(torch_cuda):
     foreground()
     for c in group:
         c.close()
+
+
+@pytest.mark.parametrize("G", [1, 4])
+@pytest.mark.parametrize("walk", [True, False])
+@pytest.mark.parametrize("key_dtype", [np.int64, np.uint32])
+def test_sparse_host_walk_parity(torch_cuda, G, walk, key_dtype):
+    """UGACHE_OPT_HOST_WALK: sparse host rows found by an input-order walk of the batch
+    (and the bucket path when off) give the oracle's bytes, with duplicates and bad keys."""
+    N, R = 400_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(31).permutation(N)]
+    t, group = make_group(torch_cuda, N, R, 20_000, G, h)
+    rng = np.random.default_rng(32)
+    keys = np.concatenate([rng.integers(0, N, 3000), rng.integers(0, 200, 20_000)])
+    rng.shuffle(keys)
+    keys[::101] = N + 3
+    for g, c in enumerate(group):
+        c.set_host_walk(walk)
+        per = check_batch(torch_cuda, c, t, keys, N, R, G, key_dtype=key_dtype)
+        assert 0 < per[G] < 4096
+    for c in group:
+        c.close()
