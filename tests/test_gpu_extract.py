@@ -469,7 +469,8 @@ def test_sparse_host_walk_parity(torch_cuda, G, walk, key_dtype):
     h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(31).permutation(N)]
     t, group = make_group(torch_cuda, N, R, 20_000, G, h)
     rng = np.random.default_rng(32)
-    keys = np.concatenate([rng.integers(0, N, 3000), rng.integers(0, 200, 20_000)])
+    hot = np.argsort(-h, kind="stable")[:15_000]          # cached somewhere (C = 20K per GPU)
+    keys = np.concatenate([rng.integers(0, N, 3000), rng.choice(hot, 20_000)])
     rng.shuffle(keys)
     keys[::101] = N + 3
     for g, c in enumerate(group):
