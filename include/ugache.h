@@ -256,8 +256,12 @@ typedef enum {
   UGACHE_OPT_DEDICATION = 3,
   UGACHE_OPT_WARP_HOST = 4,
   UGACHE_OPT_WARP_PEER = 5,
-  UGACHE_OPT_HOST_WALK = 6
+  UGACHE_OPT_HOST_WALK = 6,
+  UGACHE_OPT_FUSED = 7
 } ugache_option;
+/* UGACHE_OPT_FUSED: 0 = locate+bucket and gather as two launches; 1 = one cooperative
+ * launch (grid barrier between the phases); 2 (default) = fused for batches of up to 2^20
+ * keys.  Timing (ugache_last_batch_timing) reports the fused launch as gather time. */
 typedef enum { UGACHE_DEDICATE_SMS = 0, UGACHE_DEDICATE_WARPS = 1 } ugache_dedication;
 ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value);
 

@@ -43,7 +43,7 @@ struct Ctrl {
   uint32_t stat_bad;
   uint32_t host_arrive[2];  // intra-role barriers of the host CTAs
   uint32_t host_cursor;     // dynamic cursor over the range-ordered host bucket
-  uint32_t pad;
+  uint32_t grid_arrive;     // grid barrier of the fused locate+gather kernel
 };
 
 // Host-bucket range ordering: host rows are read in ascending
@@ -205,6 +205,7 @@ __device__ __forceinline__ void finish_launch(Ctrl *ctrl, int num_src) {
       c->host_arrive[0] = 0;
       c->host_arrive[1] = 0;
       c->host_cursor = 0;
+      c->grid_arrive = 0;
       __threadfence();
       c->done = 0;
     }
@@ -212,27 +213,28 @@ __device__ __forceinline__ void finish_launch(Ctrl *ctrl, int num_src) {
 }
 
 // ---------------------------------------------------------------------------- K1
-template <typename KeyT>
-__global__ void __launch_bounds__(kLocateThreads)
-    locate_bucket_kernel(const LocateParams p) {
-  __shared__ uint32_t s_cnt[kMaxSrc];
-  __shared__ uint32_t s_base[kMaxSrc];
+// One tile of K1 (THREADS x kLocateItems keys) processed by one CTA.  s_cnt / s_base are
+// shared arrays of kMaxSrc entries; the function starts and ends with a CTA barrier.
+template <typename KeyT, int THREADS>
+__device__ __forceinline__ void locate_tile(const LocateParams &p, uint64_t tile,
+                                            uint32_t *s_cnt, uint32_t *s_base) {
   const int tid = threadIdx.x, lane = tid & 31;
+  __syncthreads();
   if (tid < kMaxSrc) s_cnt[tid] = 0;
   __syncthreads();
   const KeyT *keys = static_cast<const KeyT *>(p.keys);
-  const uint64_t tile0 = (uint64_t)blockIdx.x * kLocateTile;
+  const uint64_t tile0 = tile * (uint64_t)(THREADS * kLocateItems);
 
   KeyT k[kLocateItems];
   uint64_t e[kLocateItems];
 #pragma unroll
   for (int it = 0; it < kLocateItems; ++it) {  // coalesced key loads
-    const uint64_t i = tile0 + (uint64_t)it * kLocateThreads + tid;
+    const uint64_t i = tile0 + (uint64_t)it * THREADS + tid;
     k[it] = (i < p.n) ? keys[i] : (KeyT)0;
   }
 #pragma unroll
   for (int it = 0; it < kLocateItems; ++it) {  // random location-table reads, all in flight
-    const uint64_t i = tile0 + (uint64_t)it * kLocateThreads + tid;
+    const uint64_t i = tile0 + (uint64_t)it * THREADS + tid;
     e[it] = (i < p.n && key_in_range<KeyT>(k[it], p.num_rows)) ? ld_nc_u64(p.loc + (uint64_t)k[it])
                                                                : ~0ull;
   }
@@ -241,7 +243,7 @@ __global__ void __launch_bounds__(kLocateThreads)
   uint32_t nbad = 0;
 #pragma unroll
   for (int it = 0; it < kLocateItems; ++it) {
-    const uint64_t i = tile0 + (uint64_t)it * kLocateThreads + tid;
+    const uint64_t i = tile0 + (uint64_t)it * THREADS + tid;
     int s = -1;
     if (i < p.n) {
       if (e[it] != ~0ull) {
@@ -267,12 +269,20 @@ __global__ void __launch_bounds__(kLocateThreads)
 #pragma unroll
   for (int it = 0; it < kLocateItems; ++it) {
     if (src[it] >= 0) {
-      const uint64_t i = tile0 + (uint64_t)it * kLocateThreads + tid;
+      const uint64_t i = tile0 + (uint64_t)it * THREADS + tid;
       const uint32_t row = (uint32_t)(e[it] & UGACHE_LOC_ROW_MASK);
       p.buckets[(uint64_t)src[it] * p.bucket_cap + s_base[src[it]] + pos[it]] =
           ((uint64_t)row << 32) | (uint64_t)i;
     }
   }
+}
+
+template <typename KeyT>
+__global__ void __launch_bounds__(kLocateThreads)
+    locate_bucket_kernel(const LocateParams p) {
+  __shared__ uint32_t s_cnt[kMaxSrc];
+  __shared__ uint32_t s_base[kMaxSrc];
+  locate_tile<KeyT, kLocateThreads>(p, blockIdx.x, s_cnt, s_base);
 }
 
 // Barrier among the `n` CTAs of one role.  The gather kernel is launched cooperatively
@@ -403,9 +413,7 @@ __device__ __forceinline__ void stride_copy(const GatherParams &p, const uint64_
 }
 
 // ---------------------------------------------------------------------------- K2
-__global__ void __launch_bounds__(kGatherThreads, 1)
-    factored_gather_kernel(const GatherParams p) {
-  extern __shared__ __align__(16) uint32_t s_dyn[];
+__device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_dyn) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   // Role of this CTA = role of the SM it runs on (one CTA per SM, cooperative launch):
   // the B200 replacement of the paper's MPS core limits.  SMs are taken in
@@ -514,6 +522,30 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
     }
   }
   finish_launch(p.ctrl, p.num_src);
+}
+
+__global__ void __launch_bounds__(kGatherThreads, 1)
+    factored_gather_kernel(const GatherParams p) {
+  extern __shared__ __align__(16) uint32_t s_dyn[];
+  gather_body(p, s_dyn);
+}
+
+// ---------------------------------------------------------------------------- K1+K2 fused
+// One cooperative launch per batch: every CTA locates + buckets tiles of 512 x 8 keys, a
+// grid-wide barrier publishes the buckets and counts, then the same CTAs run the factored
+// gather.  Saves a launch and the inter-kernel gap for small batches (DLR-shaped).
+template <typename KeyT>
+__global__ void __launch_bounds__(kGatherThreads, 1)
+    fused_extract_kernel(const LocateParams lp, const GatherParams gp) {
+  extern __shared__ __align__(16) uint32_t s_dyn[];
+  __shared__ uint32_t s_cnt[kMaxSrc];
+  __shared__ uint32_t s_base[kMaxSrc];
+  constexpr uint32_t kTile = kGatherThreads * kLocateItems;
+  const uint32_t ntiles = (lp.n + kTile - 1) / kTile;
+  for (uint32_t t = blockIdx.x; t < ntiles; t += gridDim.x)
+    locate_tile<KeyT, kGatherThreads>(lp, t, s_cnt, s_base);
+  role_barrier(&gp.ctrl->grid_arrive, gridDim.x);
+  gather_body(gp, s_dyn);
 }
 
 // ---------------------------------------------------------------------------- K2'

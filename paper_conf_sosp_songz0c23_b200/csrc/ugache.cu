@@ -68,6 +68,7 @@ struct ugache_ctx {
   int wd_host_warps = 1, wd_peer_warps = 1;  // warp-granular dedication: warps per SM
   int host_rows = ugk::kRowsInFlight;        // env UGACHE_HOST_ROWS (1, 2, 4, 8)
   int host_walk = 1;                         // UGACHE_OPT_HOST_WALK
+  int fused = 2;                             // UGACHE_OPT_FUSED: 0 off, 1 on, 2 auto
   int host_warps = ugk::kHostWarps;  // env UGACHE_HOST_WARPS (A0 calibration knob)
   int stage_host_io = 0;             // env UGACHE_STAGE_HOST_IO=1: stage pinned host I/O too
   std::vector<int> smids;  // sorted %smid values of the device (one per SM)
@@ -89,6 +90,8 @@ namespace {
 // Dynamic shared memory requested only to guarantee one gather CTA per SM, so that the
 // CTA index -> role mapping is also an SM -> role mapping (P:1620-1627 used MPS for this).
 constexpr size_t kOneCtaPerSmSmem = 120 * 1024;
+// UGACHE_OPT_FUSED = auto: batches up to this many keys run K1 + K2 in one launch.
+constexpr uint64_t kFusedAutoMaxKeys = 1u << 20;
 
 std::mutex g_reg_mu;
 std::map<const void *, int> g_reg_count;  // host-table registrations owned by this library
@@ -388,6 +391,10 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
     }
   }
   UG_CUDA(ctx, cudaFuncSetAttribute(ugk::factored_gather_kernel,
+                                    cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem));
+  UG_CUDA(ctx, cudaFuncSetAttribute(ugk::fused_extract_kernel<int64_t>,
+                                    cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem));
+  UG_CUDA(ctx, cudaFuncSetAttribute(ugk::fused_extract_kernel<uint32_t>,
                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem));
   UG_CUDA(ctx, cudaFuncSetAttribute(ugk::random_dispatch_kernel<int64_t>,
                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem));
@@ -734,6 +741,10 @@ ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value) 
       ctx->host_warps = (int)value;
       return UGACHE_OK;
     case UGACHE_OPT_HOST_WALK: ctx->host_walk = value != 0; return UGACHE_OK;
+    case UGACHE_OPT_FUSED:
+      if (value < 0 || value > 2) return UGACHE_EINVAL;
+      ctx->fused = (int)value;
+      return UGACHE_OK;
     case UGACHE_OPT_DEDICATION:
       if (value != UGACHE_DEDICATE_SMS && value != UGACHE_DEDICATE_WARPS) return UGACHE_EINVAL;
       ctx->warp_dedication = value == UGACHE_DEDICATE_WARPS;
@@ -829,15 +840,6 @@ ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type
     lp.n = (uint32_t)n;
     lp.row_bytes = R;
     lp.num_src = ctx->cfg.num_gpus + 1;
-    const unsigned lgrid = (unsigned)((n + ugk::kLocateTile - 1) / ugk::kLocateTile);
-    if (ctx->timing) UG_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
-    if (key_type == UGACHE_KEY_I64)
-      ugk::locate_bucket_kernel<int64_t><<<lgrid, ugk::kLocateThreads, 0, s>>>(lp);
-    else
-      ugk::locate_bucket_kernel<uint32_t><<<lgrid, ugk::kLocateThreads, 0, s>>>(lp);
-    UG_CUDA(ctx, cudaGetLastError());
-    if (ctx->timing) UG_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
-
     ugk::GatherParams gp;
     gp.buckets = ctx->d_buckets;
     gp.ctrl = ctx->d_ctrl;
@@ -862,10 +864,32 @@ ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type
     gp.host_warps = ctx->host_warps;
     int grid = 0;
     build_roles(ctx, &gp, &grid);
-    void *kargs[] = {&gp};
-    UG_CUDA(ctx, cudaLaunchCooperativeKernel((const void *)ugk::factored_gather_kernel, dim3(grid),
-                                             dim3(ugk::kGatherThreads), kargs, kOneCtaPerSmSmem, s));
-    ctx->last_launches = 2;
+    const bool fused = ctx->fused == 1 || (ctx->fused == 2 && n <= kFusedAutoMaxKeys);
+    if (fused) {  // K1 + K2 in one cooperative launch
+      if (ctx->timing) {
+        UG_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
+        UG_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
+      }
+      void *kargs[] = {&lp, &gp};
+      const void *fn = key_type == UGACHE_KEY_I64 ? (const void *)ugk::fused_extract_kernel<int64_t>
+                                                  : (const void *)ugk::fused_extract_kernel<uint32_t>;
+      UG_CUDA(ctx, cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(ugk::kGatherThreads), kargs,
+                                               kOneCtaPerSmSmem, s));
+      ctx->last_launches = 1;
+    } else {
+      const unsigned lgrid = (unsigned)((n + ugk::kLocateTile - 1) / ugk::kLocateTile);
+      if (ctx->timing) UG_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
+      if (key_type == UGACHE_KEY_I64)
+        ugk::locate_bucket_kernel<int64_t><<<lgrid, ugk::kLocateThreads, 0, s>>>(lp);
+      else
+        ugk::locate_bucket_kernel<uint32_t><<<lgrid, ugk::kLocateThreads, 0, s>>>(lp);
+      UG_CUDA(ctx, cudaGetLastError());
+      if (ctx->timing) UG_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
+      void *kargs[] = {&gp};
+      UG_CUDA(ctx, cudaLaunchCooperativeKernel((const void *)ugk::factored_gather_kernel, dim3(grid),
+                                               dim3(ugk::kGatherThreads), kargs, kOneCtaPerSmSmem, s));
+      ctx->last_launches = 2;
+    }
   }
   if (ctx->timing) {
     UG_CUDA(ctx, cudaEventRecord(ctx->ev[2], s));

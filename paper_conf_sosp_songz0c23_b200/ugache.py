@@ -189,6 +189,10 @@ class UGache:
         if peer_warps:
             self.set_option(_abi.OPT_WARP_PEER, peer_warps)
 
+    def set_fused(self, mode):
+        """'off' (two launches), 'on' (one cooperative launch) or 'auto'."""
+        self.set_option(_abi.OPT_FUSED, {"off": 0, "on": 1, "auto": 2}[mode])
+
     def set_host_walk(self, on: bool):
         self.set_option(_abi.OPT_HOST_WALK, int(on))
 
