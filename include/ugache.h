@@ -211,16 +211,19 @@ ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type
  *   1. ugache_refresh_begin(new placement): every key whose location changes is pointed at
  *      the host now (async on stream); extracts stay correct and simply read those keys
  *      from host DRAM.   -> all GPUs, then >= 1 foreground batch + barrier
- *   2. ugache_refresh_content(max_sms): rewrite the slots whose key changes from the host
- *      table (only those), using at most max_sms SMs' worth of CTAs (0 = all; throttling,
- *      P:1611-1616); synchronous.   -> all GPUs, then barrier
+ *   2. ugache_refresh_content(max_sms, max_rows, &remaining): rewrite the slots whose key
+ *      changes from the host table (only those), at most max_rows per call (0 = all) with
+ *      at most max_sms SMs' worth of CTAs (0 = all) -- the refresh granularity / resource
+ *      throttle of P:1611-1616; synchronous; call again while remaining > 0 (foreground
+ *      batches may run in between).   -> all GPUs, then barrier
  *   3. ugache_refresh_commit: install the new location table and slot list.
  * new_loc / new_slot_keys: as for ugache_init_with_placement (checked the same way).  Not
  * available with UGACHE_FLAG_HOST_TIER.  Wrong order -> ESTATE. */
 ugache_status ugache_refresh_begin(ugache_ctx *ctx, const uint64_t *new_loc,
                                    const uint64_t *new_slot_keys, uint64_t n_new_slots,
                                    void *stream);
-ugache_status ugache_refresh_content(ugache_ctx *ctx, int32_t max_sms, void *stream);
+ugache_status ugache_refresh_content(ugache_ctx *ctx, int32_t max_sms, uint64_t max_rows,
+                                     uint64_t *remaining, void *stream);
 ugache_status ugache_refresh_commit(ugache_ctx *ctx, void *stream);
 
 /* Core dedication override: SMs for host and for each peer; local gets the

@@ -81,7 +81,7 @@ SIGNATURES = {
     "ugache_fill": (_ST, [_P, _P]),
     "ugache_extract": (_ST, [_P, _P, _c.c_int32, _c.c_uint64, _P, _P]),
     "ugache_refresh_begin": (_ST, [_P, _P, _P, _c.c_uint64, _P]),
-    "ugache_refresh_content": (_ST, [_P, _c.c_int32, _P]),
+    "ugache_refresh_content": (_ST, [_P, _c.c_int32, _c.c_uint64, ctypes.POINTER(_c.c_uint64), _P]),
     "ugache_refresh_commit": (_ST, [_P, _P]),
     "ugache_set_dedication": (_ST, [_P, _c.c_int32, _c.c_int32]),
     "ugache_set_mode": (_ST, [_P, _c.c_int32]),

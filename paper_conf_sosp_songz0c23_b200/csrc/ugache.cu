@@ -44,7 +44,8 @@ struct ugache_ctx {
   int refresh_state = 0;
   uint64_t *d_loc_new = nullptr;
   std::vector<uint64_t> new_slot_keys;
-  uint64_t refresh_changed = 0;
+  uint64_t refresh_changed = 0, refresh_pos = 0;
+  uint64_t *d_refresh = nullptr;  // changed (slot, key) lists staged for the content step
   // sources
   const uint8_t *src_base[ug::kMaxSrc] = {};
   void *ipc_mapped[UGACHE_MAX_GPUS] = {};
@@ -641,44 +642,53 @@ ugache_status ugache_refresh_begin(ugache_ctx *ctx, const uint64_t *new_loc,
   return UGACHE_OK;
 }
 
-ugache_status ugache_refresh_content(ugache_ctx *ctx, int32_t max_sms, void *stream) {
+ugache_status ugache_refresh_content(ugache_ctx *ctx, int32_t max_sms, uint64_t max_rows,
+                                     uint64_t *remaining, void *stream) {
   if (!ctx || max_sms < 0) return UGACHE_EINVAL;
   if (ctx->refresh_state != 1) return fail(ctx, UGACHE_ESTATE, "refresh_content before refresh_begin");
   ugache_status st = begin(ctx);
   if (st != UGACHE_OK) return st;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
-  std::vector<uint64_t> idx, keys;
-  for (uint64_t i = 0; i < ctx->new_slot_keys.size(); ++i)
-    if (i >= ctx->h_slot_keys.size() || ctx->h_slot_keys[i] != ctx->new_slot_keys[i]) {
-      idx.push_back(i);
-      keys.push_back(ctx->new_slot_keys[i]);
+  if (!ctx->d_refresh) {  // first call: the changed slots, staged on the device once
+    std::vector<uint64_t> idx, keys;
+    for (uint64_t i = 0; i < ctx->new_slot_keys.size(); ++i)
+      if (i >= ctx->h_slot_keys.size() || ctx->h_slot_keys[i] != ctx->new_slot_keys[i]) {
+        idx.push_back(i);
+        keys.push_back(ctx->new_slot_keys[i]);
+      }
+    ctx->refresh_changed = idx.size();
+    ctx->refresh_pos = 0;
+    UG_CUDA(ctx, cudaMalloc(&ctx->d_refresh, 2 * std::max<size_t>(idx.size(), 1) * sizeof(uint64_t)));
+    if (!idx.empty()) {
+      UG_CUDA(ctx, cudaMemcpy(ctx->d_refresh, idx.data(), idx.size() * 8, cudaMemcpyHostToDevice));
+      UG_CUDA(ctx, cudaMemcpy(ctx->d_refresh + idx.size(), keys.data(), keys.size() * 8,
+                              cudaMemcpyHostToDevice));
     }
-  ctx->refresh_changed = idx.size();
-  if (!idx.empty()) {
-    uint64_t *d = nullptr;
-    UG_CUDA(ctx, cudaMalloc(&d, 2 * idx.size() * sizeof(uint64_t)));
-    cudaError_t e = cudaMemcpy(d, idx.data(), idx.size() * 8, cudaMemcpyHostToDevice);
-    if (e == cudaSuccess) e = cudaMemcpy(d + idx.size(), keys.data(), keys.size() * 8, cudaMemcpyHostToDevice);
-    if (e != cudaSuccess) {
-      cudaFree(d);
-      return cuda_fail(ctx, e, "refresh staging");
-    }
+  }
+  const uint64_t total = ctx->refresh_changed;
+  const uint64_t lo = ctx->refresh_pos;
+  const uint64_t hi = max_rows ? std::min(total, lo + max_rows) : total;
+  if (hi > lo) {
     ugk::FillParams fp;
-    fp.slot_idx = d;
-    fp.slot_keys = d + idx.size();
+    fp.slot_idx = ctx->d_refresh + lo;
+    fp.slot_keys = ctx->d_refresh + total + lo;
     fp.table = ctx->host_table_dev;
     fp.slab = ctx->slab;
-    fp.n_slots = idx.size();
+    fp.n_slots = hi - lo;
     fp.row_bytes = ctx->cfg.row_bytes;
-    // throttle: the refresh touches at most max_sms SMs' worth of CTAs
+    // throttle: at most max_sms SMs' worth of CTAs, max_rows rows per call
     const int sms = max_sms ? std::min(max_sms, ctx->sm_count) : ctx->sm_count;
     ugk::fill_kernel<<<sms * 8, 256, 0, s>>>(fp);
-    e = cudaGetLastError();
-    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
-    cudaFree(d);
-    if (e != cudaSuccess) return cuda_fail(ctx, e, "refresh fill");
+    UG_CUDA(ctx, cudaGetLastError());
+    UG_CUDA(ctx, cudaStreamSynchronize(s));
   }
-  ctx->refresh_state = 2;
+  ctx->refresh_pos = hi;
+  if (remaining) *remaining = total - hi;
+  if (hi == total) {
+    cudaFree(ctx->d_refresh);
+    ctx->d_refresh = nullptr;
+    ctx->refresh_state = 2;
+  }
   return UGACHE_OK;
 }
 
@@ -987,6 +997,7 @@ ugache_status ugache_destroy(ugache_ctx *ctx) {
     cudaFree(ctx->d_host_sorted);
     cudaFree(ctx->d_ranges);
     cudaFree(ctx->d_loc_new);
+    cudaFree(ctx->d_refresh);
     for (int i = 0; i < 3; ++i)
       if (ctx->ev[i]) cudaEventDestroy(ctx->ev[i]);
   }

@@ -159,9 +159,12 @@ class UGache:
         check(lib().ugache_refresh_begin(self.ctx, _ptr(loc), _ptr(sk), len(sk), _stream_handle(stream)),
               "ugache_refresh_begin", self.ctx)
 
-    def refresh_content(self, max_sms: int = 0, stream=None):
-        check(lib().ugache_refresh_content(self.ctx, max_sms, _stream_handle(stream)),
-              "ugache_refresh_content", self.ctx)
+    def refresh_content(self, max_sms: int = 0, max_rows: int = 0, stream=None) -> int:
+        """One content step; returns the number of changed slots still to rewrite."""
+        rem = ctypes.c_uint64()
+        check(lib().ugache_refresh_content(self.ctx, max_sms, max_rows, ctypes.byref(rem),
+                                           _stream_handle(stream)), "ugache_refresh_content", self.ctx)
+        return int(rem.value)
 
     def refresh_commit(self, stream=None):
         check(lib().ugache_refresh_commit(self.ctx, _stream_handle(stream)), "ugache_refresh_commit",

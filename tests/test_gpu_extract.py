@@ -436,8 +436,9 @@ def test_cache_refresh_protocol(torch_cuda):
     foreground()                                  # transitional tables
     with pytest.raises(Exception):
         group[0].refresh_commit()                 # content step missing -> ESTATE
-    for c in group:
-        c.refresh_content(max_sms=4)
+    for c in group:                               # chunked content, foreground in between
+        while c.refresh_content(max_sms=4, max_rows=700) > 0:
+            foreground()
     foreground()                                  # new content, transitional tables
     for c in group:
         c.refresh_commit()
@@ -453,7 +454,7 @@ def test_cache_refresh_protocol(torch_cuda):
             assert np.array_equal(c.read_slab(0, len(sk))[idx], t.array[sk[idx].astype(np.int64)])
     check_placement(np.stack(locs), sks, N, C)
     # refresh back with the group helper
-    refresh_group(group, pl1, max_sms=8, foreground=foreground)
+    refresh_group(group, pl1, max_sms=8, max_rows=2500, foreground=foreground)
     foreground()
     for c in group:
         c.close()
