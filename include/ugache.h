@@ -203,6 +203,32 @@ ugache_status ugache_fill(ugache_ctx *ctx, void *stream);
 ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type, uint64_t n,
                              void *out, void *stream);
 
+/* ---- message-based baseline -----------------------
+ * The design UGache argues against: "a GPU sends keys to the GPU caching them, which then
+ * looks up and sends back the values" and the requester must "reorder ... back to the
+ * original key order".  Same placement, location table and kernels as the
+ * factored path; the peer rows travel through two all-to-all exchanges done by the CALLER
+ * (NCCL via torch.distributed), never through peer loads.  Per batch, on every GPU:
+ *   1. ugache_msg_extract_local(keys, out): locate + bucket every key, copy the local and
+ *      host rows into out (peer SMs = 0); the peer buckets stay in the ctx.
+ *   2. ugache_msg_requests(counts, req): synchronises the stream, returns the per-source
+ *      key counts (G+1 entries as ugache_last_batch_stats) and packs the slot ids wanted
+ *      from each peer into req (device, >= sum of the peer counts u32 entries), peers in
+ *      rank order.  The caller exchanges counts and req (all-to-all).
+ *   3. ugache_msg_serve(req_in, n_req, send): on the owner, send[i] = slab row req_in[i]
+ *      (device buffers; n_req*R bytes).  The caller all-to-alls send back.
+ *   4. ugache_msg_scatter(replies, out): replies packed in the same peer order as req;
+ *      out[out_idx] = reply row.  out must be the out of step 1.
+ * Steps 2-4 must follow step 1 of the same batch on the same ctx with no extract in
+ * between (ESTATE otherwise).  Device memory only for req/send/replies/out.  Not for the
+ * hot path: it exists to measure the paper's message-based comparison (Fig. 4 / Fig. 13). */
+ugache_status ugache_msg_extract_local(ugache_ctx *ctx, const void *keys, int32_t key_type,
+                                       uint64_t n, void *out, void *stream);
+ugache_status ugache_msg_requests(ugache_ctx *ctx, uint64_t *counts, uint32_t *req, void *stream);
+ugache_status ugache_msg_serve(ugache_ctx *ctx, const uint32_t *req_in, uint64_t n_req, void *send,
+                               void *stream);
+ugache_status ugache_msg_scatter(ugache_ctx *ctx, const void *replies, void *out, void *stream);
+
 /* ---- cache refresh (section 7.2) ----------------------------------------
  * "Refresher evicts old entries and inserts new entries into UGache's hashtable and cache
  * content ... Refresher waits for a foreground batch between the update of hashtable and

@@ -80,6 +80,10 @@ SIGNATURES = {
     "ugache_set_peer_slabs": (_ST, [_P, ctypes.POINTER(_P)]),
     "ugache_fill": (_ST, [_P, _P]),
     "ugache_extract": (_ST, [_P, _P, _c.c_int32, _c.c_uint64, _P, _P]),
+    "ugache_msg_extract_local": (_ST, [_P, _P, _c.c_int32, _c.c_uint64, _P, _P]),
+    "ugache_msg_requests": (_ST, [_P, _P, _P, _P]),
+    "ugache_msg_serve": (_ST, [_P, _P, _c.c_uint64, _P, _P]),
+    "ugache_msg_scatter": (_ST, [_P, _P, _P, _P]),
     "ugache_refresh_begin": (_ST, [_P, _P, _P, _c.c_uint64, _P]),
     "ugache_refresh_content": (_ST, [_P, _c.c_int32, _c.c_uint64, ctypes.POINTER(_c.c_uint64), _P]),
     "ugache_refresh_commit": (_ST, [_P, _P]),

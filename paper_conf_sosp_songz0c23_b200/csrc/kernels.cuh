@@ -642,6 +642,91 @@ __global__ void __launch_bounds__(256) fill_kernel(const FillParams p) {
   }
 }
 
+// ---------------------------------------------------------------------------- message path
+// The message-based baseline ("peer-based" vs "message-based" extraction): the
+// requester sends the slot ids it needs to each owner, the owner gathers them into a
+// contiguous send buffer, the rows travel back in a collective, and the requester
+// scatters them into key order.  Only the three device steps are here; the two
+// all-to-all exchanges are the caller's (NCCL through torch.distributed).
+struct MsgSeg {
+  uint32_t src;    // peer GPU id (bucket index)
+  uint32_t count;  // entries of that bucket
+  uint64_t off;    // first entry of this peer's segment in the packed request / reply
+};
+
+struct MsgParams {
+  const uint64_t *buckets;
+  uint64_t bucket_cap;
+  MsgSeg seg[kMaxSrc];
+  int32_t n_seg;
+  uint64_t total;
+  uint32_t *req;             // pack: out, one slot id per entry
+  const uint32_t *req_in;    // serve: in
+  const uint8_t *slab;       // serve: this GPU's cache slab
+  uint64_t slab_rows;        // serve: rows >= slab_rows zero-fill (never produced by a valid LT)
+  const uint8_t *rows_in;    // scatter: replies, packed in segment order
+  uint8_t *rows_out;         // serve: send buffer / scatter: out
+  uint32_t row_bytes;
+};
+
+__device__ __forceinline__ int msg_segment(const MsgParams &p, uint64_t i) {
+  int s = 0;
+  while (s + 1 < p.n_seg && i >= p.seg[s + 1].off) ++s;
+  return s;
+}
+
+__global__ void __launch_bounds__(256) msg_pack_kernel(const MsgParams p) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < p.total;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    const MsgSeg g = p.seg[msg_segment(p, i)];
+    p.req[i] = (uint32_t)(p.buckets[(uint64_t)g.src * p.bucket_cap + (i - g.off)] >> 32);
+  }
+}
+
+// Warp per U rows: serve (slab[req[i]] -> send[i]) or scatter (reply[i] -> out[out_idx]).
+template <bool SCATTER>
+__global__ void __launch_bounds__(512) msg_copy_kernel(const MsgParams p) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t W = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  const uint32_t R = p.row_bytes, V = R >> 4;
+  for (uint64_t e0 = (((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * kRowsInFlight; e0 < p.total;
+       e0 += W * kRowsInFlight) {
+    const int nv = (int)min((uint64_t)kRowsInFlight, p.total - e0);
+    uint64_t s_row = 0, d_row = 0;
+    bool zero = false;
+    if (lane < nv) {
+      const uint64_t i = e0 + lane;
+      if (SCATTER) {
+        const MsgSeg g = p.seg[msg_segment(p, i)];
+        s_row = i;
+        d_row = p.buckets[(uint64_t)g.src * p.bucket_cap + (i - g.off)] & 0xFFFFFFFFull;
+      } else {
+        s_row = p.req_in[i];
+        d_row = i;
+        zero = s_row >= p.slab_rows;
+      }
+    }
+    const uint8_t *src = SCATTER ? p.rows_in : p.slab;
+    uint64_t su[kRowsInFlight], du[kRowsInFlight];
+    bool zu[kRowsInFlight];
+#pragma unroll
+    for (int u = 0; u < kRowsInFlight; ++u) {
+      su[u] = __shfl_sync(kFullMask, s_row, u);
+      du[u] = __shfl_sync(kFullMask, d_row, u);
+      zu[u] = __shfl_sync(kFullMask, zero, u);
+    }
+    for (uint32_t j = lane; j < V; j += 32) {
+      uint4 v[kRowsInFlight];
+#pragma unroll
+      for (int u = 0; u < kRowsInFlight; ++u)
+        if (u < nv) v[u] = zu[u] ? make_uint4(0, 0, 0, 0) : ld_nc_v4(src + su[u] * R + (uint64_t)j * 16u);
+#pragma unroll
+      for (int u = 0; u < kRowsInFlight; ++u)
+        if (u < nv) st_cs_v4(p.rows_out + du[u] * R + (uint64_t)j * 16u, v[u]);
+    }
+  }
+}
+
 // ---------------------------------------------------------------------------- refresh
 // Cache refresh, step 1: every key whose location changes is first pointed at
 // the host (which holds every entry), so no reader can reach a slot whose content is about

@@ -81,6 +81,10 @@ struct ugache_ctx {
   bool timing_valid = false;
   cudaEvent_t ev[3] = {};
   int last_launches = 0;
+  // message-based baseline: 0 idle, 1 local part done (buckets valid), 2 requests packed
+  int msg_state = 0;
+  uint64_t msg_counts[ug::kMaxSrc] = {};
+  void *msg_out = nullptr;
   uint64_t last_n = 0;
   cudaStream_t last_stream = nullptr;
   std::string err;
@@ -772,9 +776,11 @@ ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value) 
   return UGACHE_EINVAL;
 }
 
-ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type, uint64_t n,
-                             void *out, void *stream) {
+namespace {
+ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, uint64_t n,
+                           void *out, void *stream, bool msg_local) {
   if (!ctx) return UGACHE_EINVAL;
+  ctx->msg_state = 0;
   if (key_type != UGACHE_KEY_I64 && key_type != UGACHE_KEY_U32) return UGACHE_EINVAL;
   if (n >= (1ull << 32)) return UGACHE_EINVAL;
   if (!ctx->filled || !ctx->peers_ready) return fail(ctx, UGACHE_ESTATE, "extract before fill/peers");
@@ -874,6 +880,11 @@ ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type
     gp.host_warps = ctx->host_warps;
     int grid = 0;
     build_roles(ctx, &gp, &grid);
+    if (msg_local) {  // message baseline: no SM reads a peer; the peer buckets stay for msg_*
+      gp.n_peers = 0;
+      gp.peer_sms = 0;
+      gp.host_sms_max = ctx->host_dynamic ? std::max(ctx->host_sms, gp.num_sms) : ctx->host_sms;
+    }
     const bool fused = ctx->fused == 1 || (ctx->fused == 2 && n <= kFusedAutoMaxKeys);
     if (fused) {  // K1 + K2 in one cooperative launch
       if (ctx->timing) {
@@ -907,6 +918,118 @@ ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type
   }
   if (host_out) UG_CUDA(ctx, cudaMemcpyAsync(out, dout, n * (size_t)R, cudaMemcpyDeviceToHost, s));
   ctx->last_stream = s;
+  return UGACHE_OK;
+}
+}  // namespace
+
+ugache_status ugache_extract(ugache_ctx *ctx, const void *keys, int32_t key_type, uint64_t n,
+                             void *out, void *stream) {
+  return extract_impl(ctx, keys, key_type, n, out, stream, false);
+}
+
+// ---------------------------------------------------------------- message-based baseline
+ugache_status ugache_msg_extract_local(ugache_ctx *ctx, const void *keys, int32_t key_type,
+                                       uint64_t n, void *out, void *stream) {
+  if (!ctx) return UGACHE_EINVAL;
+  if (ctx->mode != UGACHE_MODE_FACTORED) return fail(ctx, UGACHE_ESTATE, "message path needs the factored mode");
+  void *unused = nullptr;
+  if (n && out && mem_kind(out, &unused) != MemKind::kDevice)
+    return fail(ctx, UGACHE_EINVAL, "message path: out must be device memory");
+  ugache_status st = extract_impl(ctx, keys, key_type, n, out, stream, true);
+  if (st != UGACHE_OK) return st;
+  ctx->msg_state = 1;
+  ctx->msg_out = out;
+  return UGACHE_OK;
+}
+
+namespace {
+void msg_segments(const ugache_ctx *ctx, ugk::MsgParams *mp) {
+  const int G = ctx->cfg.num_gpus, me = ctx->cfg.rank;
+  mp->buckets = ctx->d_buckets;
+  mp->bucket_cap = ctx->bucket_cap;
+  mp->n_seg = 0;
+  uint64_t off = 0;
+  for (int j = 0; j < G; ++j) {
+    if (j == me) continue;
+    mp->seg[mp->n_seg].src = (uint32_t)j;
+    mp->seg[mp->n_seg].count = (uint32_t)ctx->msg_counts[j];
+    mp->seg[mp->n_seg].off = off;
+    off += ctx->msg_counts[j];
+    ++mp->n_seg;
+  }
+  mp->total = off;
+  mp->row_bytes = ctx->cfg.row_bytes;
+}
+unsigned msg_grid(const ugache_ctx *ctx, uint64_t rows_or_items, unsigned per_block) {
+  const uint64_t b = (rows_or_items + per_block - 1) / per_block;
+  return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(b, (uint64_t)ctx->sm_count * 8));
+}
+}  // namespace
+
+ugache_status ugache_msg_requests(ugache_ctx *ctx, uint64_t *counts, uint32_t *req, void *stream) {
+  if (!ctx || !counts) return UGACHE_EINVAL;
+  if (ctx->msg_state != 1) return fail(ctx, UGACHE_ESTATE, "msg_requests without msg_extract_local");
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  const int S = ctx->cfg.num_gpus + 1;
+  if (ctx->last_n == 0 || ctx->last_launches == 0) {
+    for (int j = 0; j < S; ++j) ctx->msg_counts[j] = 0;
+  } else {
+    UG_CUDA(ctx, cudaStreamSynchronize(ctx->last_stream));
+    ugk::Ctrl c;
+    UG_CUDA(ctx, cudaMemcpy(&c, ctx->d_ctrl, sizeof(c), cudaMemcpyDeviceToHost));
+    for (int j = 0; j < S; ++j) ctx->msg_counts[j] = c.stat_counts[j];
+  }
+  for (int j = 0; j < S; ++j) counts[j] = ctx->msg_counts[j];
+  ugk::MsgParams mp{};
+  msg_segments(ctx, &mp);
+  mp.req = req;
+  if (mp.total) {
+    if (!req) return UGACHE_EINVAL;
+    ugk::msg_pack_kernel<<<msg_grid(ctx, mp.total, 256), 256, 0, static_cast<cudaStream_t>(stream)>>>(mp);
+    UG_CUDA(ctx, cudaGetLastError());
+  }
+  ctx->msg_state = 2;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_msg_serve(ugache_ctx *ctx, const uint32_t *req_in, uint64_t n_req, void *send,
+                               void *stream) {
+  if (!ctx) return UGACHE_EINVAL;
+  if (!n_req) return UGACHE_OK;
+  if (!req_in || !send) return UGACHE_EINVAL;
+  if (!ctx->filled) return fail(ctx, UGACHE_ESTATE, "serve before fill");
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  ugk::MsgParams mp{};
+  mp.total = n_req;
+  mp.req_in = req_in;
+  mp.slab = ctx->slab;
+  mp.slab_rows = ctx->plan.capacity_rows;
+  mp.rows_out = static_cast<uint8_t *>(send);
+  mp.row_bytes = ctx->cfg.row_bytes;
+  ugk::msg_copy_kernel<false><<<msg_grid(ctx, n_req, 16 * ugk::kRowsInFlight), 512, 0,
+                                static_cast<cudaStream_t>(stream)>>>(mp);
+  UG_CUDA(ctx, cudaGetLastError());
+  return UGACHE_OK;
+}
+
+ugache_status ugache_msg_scatter(ugache_ctx *ctx, const void *replies, void *out, void *stream) {
+  if (!ctx) return UGACHE_EINVAL;
+  if (ctx->msg_state != 2) return fail(ctx, UGACHE_ESTATE, "msg_scatter without msg_requests");
+  if (out != ctx->msg_out) return fail(ctx, UGACHE_EINVAL, "msg_scatter: out differs from msg_extract_local's");
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  ugk::MsgParams mp{};
+  msg_segments(ctx, &mp);
+  ctx->msg_state = 0;
+  if (!mp.total) return UGACHE_OK;
+  if (!replies || !out) return UGACHE_EINVAL;
+  mp.rows_in = static_cast<const uint8_t *>(replies);
+  mp.rows_out = static_cast<uint8_t *>(out);
+  ugk::msg_copy_kernel<true><<<msg_grid(ctx, mp.total, 16 * ugk::kRowsInFlight), 512, 0,
+                               static_cast<cudaStream_t>(stream)>>>(mp);
+  UG_CUDA(ctx, cudaGetLastError());
   return UGACHE_OK;
 }
 

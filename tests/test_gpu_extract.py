@@ -498,3 +498,40 @@ def test_fused_and_split_launch_parity(torch_cuda, fused, G, C, n):
             assert c.last_launch_count() == (1 if fused == "on" else 2)
     for c in group:
         c.close()
+
+
+@pytest.mark.parametrize("G,policy", [(1, "ugache"), (2, "partition"), (4, "ugache"), (8, "partition")])
+@pytest.mark.parametrize("fused", ["on", "off"])
+def test_message_based_baseline_parity(torch_cuda, G, policy, fused):
+    """Message-based baseline: local/host rows by the factored kernels with no
+    peer SMs, peer rows through request/serve/reply exchanges and a scatter into key order
+     -- same bytes and per-source counts as the oracle, incl. out-of-range keys."""
+    from paper_conf_sosp_songz0c23_b200.message import message_extract_group
+    wl = synth.get_workload("tiny")
+    h = synth.hotness(wl)
+    N, R = wl.num_rows, wl.row_bytes
+    t, group = make_group(torch_cuda, N, R, 4000, G, h, policy=policy)
+    for c in group:
+        c.set_fused(fused)
+    for b in range(2):
+        keys_np = [synth.make_batch(wl, g, b) for g in range(G)]
+        keys_np[0][::777] = N + 3
+        keys = [torch_cuda.from_numpy(k).cuda() for k in keys_np]
+        outs = message_extract_group(group, keys)
+        torch_cuda.cuda.synchronize()
+        for g, c in enumerate(group):
+            ref, bad = oracle.gather(t.ptr, N, R, keys_np[g])
+            assert np.array_equal(outs[g].cpu().numpy(), ref)
+            per, nbad = c.last_batch_stats()
+            loc, _ = c.export_placement()
+            ref_cnt, ref_bad = source_counts(loc, keys_np[g], N, G)
+            assert nbad == ref_bad == bad and np.array_equal(per, ref_cnt)
+            if G > 1 and b == 0:
+                assert per[[j for j in range(G) if j != g]].sum() > 0
+    # protocol misuse: scatter without the earlier steps -> ESTATE
+    from paper_conf_sosp_songz0c23_b200._abi import UGacheError
+    from paper_conf_sosp_songz0c23_b200 import message
+    with pytest.raises(UGacheError):
+        message._scatter(group[0], outs[0], outs[0], None)
+    for c in group:
+        c.close()
