@@ -423,11 +423,18 @@ def main():
     n_local = float(per[rank]) if G > 0 else 0.0
     n_host = float(per[G])
     n_peer = float(per.sum() - n_local - n_host)
-    kb = 8
-    gat_s = statistics.mean(gat_ms) / 1e3
+    kb = 8 if dkeys[0].dtype == torch.int64 else 4
+    # the timed kernel: K2 alone (two launches) or the whole fused K1+K2 launch
+    kern_ms = [a + b for a, b in zip(loc_ms, gat_ms)] if launches == args.steps else list(gat_ms)
+    gat_s = statistics.mean(kern_ms) / 1e3
     loc_s = statistics.mean(loc_ms) / 1e3
-    # algorithmic bytes of the gather kernel: rows read per source + rows written + bucket reads
-    gather_hbm_bytes = n_local * R + n * R + n * 8
+    # algorithmic bytes of the timed kernel: rows read per source + rows written + bucket
+    # reads; with K1+K2 fused (one launch per step) also K1's key + location entry + bucket
+    # write per key (2R + 8 + 8 + 16 per key)
+    fused = launches == args.steps
+    kname = "fused_extract_kernel" if fused else "factored_gather_kernel"
+    k1_hbm_bytes = n * (kb + 8 + 8)
+    gather_hbm_bytes = n_local * R + n * R + n * 8 + (k1_hbm_bytes if fused else 0)
     gather_pcie_bytes = n_host * R
     t_hbm = gather_hbm_bytes / (hbm * 1e9)
     t_pcie = gather_pcie_bytes / (pcie * 1e9) if pcie else 0.0
@@ -444,13 +451,13 @@ def main():
         achieved, peak, unit, psrc = n_peer * R / gat_s / 1e9, nvl, "GB/s", \
             "B200_PROFILING.md measured peer copy"
     # whole-step source-mix roofline (locate + gather): every byte the step moves
-    step_hbm = (n * kb + n * 32 + n * 8 + n * 8) + gather_hbm_bytes
+    step_hbm = n_local * R + n * R + n * 8 + k1_hbm_bytes
     t_roof = max(step_hbm / (hbm * 1e9), t_pcie, t_nvl)
     ms_per_step = statistics.mean(step_ms)
     traffic = traffic_pcie = traffic_src = None
     try:  # per-launch DRAM traffic of K2 from the committed ncu capture of this workload
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
-            rec = json.load(f)[wl.name]["factored_gather_kernel"]
+            rec = json.load(f)[wl.name][kname]
         traffic, traffic_pcie, traffic_src = rec["dram_bytes"], rec.get("pcie_read_bytes"), rec["source"]
     except Exception:
         pass
@@ -464,8 +471,9 @@ def main():
                      "traffic_pcie_read": traffic_pcie, "traffic_source": traffic_src,
                      "algorithmic_bytes": {"hbm": gather_hbm_bytes, "pcie": gather_pcie_bytes,
                                            "nvlink": n_peer * R},
-                     "kernel": "factored_gather_kernel", "peak_source": psrc,
-                     "kernel_ms": statistics.mean(gat_ms)},
+                     "kernel": kname + (" (K1 locate+bucket and K2 gather, one cooperative launch)" if fused else ""),
+                     "peak_source": psrc,
+                     "kernel_ms": statistics.mean(kern_ms)},
         "source_mix_roofline": {"t_roof_us": t_roof * 1e6, "t_step_us": ms_per_step * 1e3,
                                 "frac": t_roof / (ms_per_step / 1e3),
                                 "terms_us": {"hbm": step_hbm / (hbm * 1e9) * 1e6,

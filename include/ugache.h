@@ -286,11 +286,19 @@ typedef enum {
   UGACHE_OPT_WARP_HOST = 4,
   UGACHE_OPT_WARP_PEER = 5,
   UGACHE_OPT_HOST_WALK = 6,
-  UGACHE_OPT_FUSED = 7
+  UGACHE_OPT_FUSED = 7,
+  UGACHE_OPT_LOCAL_BULK = 8
 } ugache_option;
-/* UGACHE_OPT_FUSED: 0 = locate+bucket and gather as two launches; 1 = one cooperative
+/* UGACHE_OPT_LOCAL_BULK: local rows (A4) move HBM -> shared -> HBM as TMA cp.async.bulk
+ *   copies (no registers per row, ~196 KB in flight per SM) instead of LDG.128 / STG.128
+ *   through registers.  0 = never, 1 = always, 2 (default) = unless the host bucket is
+ *   dense enough for range-ordered reads (a PCIe-bound batch, where the register path's
+ *   local burst interferes less with the host reads), 3 = on CTAs without a host role.
+ *   Rows larger than 6 KB always use the register path.
+ * UGACHE_OPT_FUSED: 0 = locate+bucket and gather as two launches; 1 = one cooperative
  * launch (grid barrier between the phases); 2 (default) = fused for batches of up to 2^20
- * keys.  Timing (ugache_last_batch_timing) reports the fused launch as gather time. */
+ * keys.  Timing (ugache_last_batch_timing) splits the fused launch at its grid barrier
+ * (device %globaltimer stamps): locate = start .. barrier, gather = the rest. */
 typedef enum { UGACHE_DEDICATE_SMS = 0, UGACHE_DEDICATE_WARPS = 1 } ugache_dedication;
 ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value);
 

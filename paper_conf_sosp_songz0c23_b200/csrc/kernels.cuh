@@ -44,7 +44,15 @@ struct Ctrl {
   uint32_t host_arrive[2];  // intra-role barriers of the host CTAs
   uint32_t host_cursor;     // dynamic cursor over the range-ordered host bucket
   uint32_t grid_arrive;     // grid barrier of the fused locate+gather kernel
+  unsigned long long t_start;    // fused kernel: %globaltimer at CTA 0's start (ns)
+  unsigned long long t_located;  // fused kernel: %globaltimer when CTA 0 leaves the grid barrier
 };
+
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
 
 // Host-bucket range ordering: host rows are read in ascending
 // key-range order so that the rows in flight span a small window of host address space
@@ -52,6 +60,13 @@ struct Ctrl {
 constexpr int kMaxRanges = 4096;
 constexpr uint32_t kHostSortMin = 4096;  // never order fewer host keys than this
 constexpr int kRowsPerSmRound = kGatherWarps * kRowsInFlight;  // rows one SM keeps in flight
+
+// Dynamic shared memory of the gather kernels: [host range table | per-warp bulk slots].
+// Its size (> half of the SM's 228 KB) also guarantees one gather CTA per SM.
+constexpr uint32_t kRangeTabBytes = kMaxRanges * 4;
+constexpr uint32_t kBulkWarpBytes = 12 * 1024;          // TMA staging per warp (24 rows of 512 B)
+constexpr int kBulkMaxSlots = 32;                       // slots (rows) per warp
+constexpr uint32_t kGatherSmem = kRangeTabBytes + kGatherWarps * kBulkWarpBytes;  // 208 KB
 
 struct LocateParams {
   const void *keys;
@@ -103,6 +118,8 @@ struct GatherParams {
   uint32_t n_keys;
   int32_t keys_u32;                // key type: 0 = int64, 1 = uint32
   int32_t host_walk;               // 1 = sparse host buckets use the input-order walk
+  int32_t local_bulk;              // local rows by TMA bulk copies: 0 never, 1 always, 2 unless
+                                   // the host bucket is dense, 3 on CTAs without a host role
 };
 
 struct RandomParams {
@@ -412,6 +429,112 @@ __device__ __forceinline__ void stride_copy(const GatherParams &p, const uint64_
   }
 }
 
+// ---------------------------------------------------------------------------- TMA bulk
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+  uint32_t done = 0;
+  while (!done) {
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+  }
+}
+// global -> shared, completion counted on bar (bytes multiple of 16, 16-B aligned)
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+// shared -> global, tracked by this thread's bulk groups; policy: an L2 cache policy
+// (evict_first for the output stream, like st.global.cs on the register path)
+__device__ __forceinline__ void bulk_s2g(void *dst, const void *src, uint32_t bytes, uint64_t policy) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;" ::"l"(dst),
+               "r"(smem_u32(src)), "r"(bytes), "l"(policy)
+               : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ uint64_t l2_evict_first_policy() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+__device__ __forceinline__ void bulk_wait_read_all() {
+  asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// Local bucket drained by TMA bulk copies (A4 on B200): each row goes HBM -> shared memory
+// -> HBM as two cp.async.bulk operations, no registers hold row data, so one SM keeps
+// 16 warps x 24 rows = 196 KB in flight (LDG.128 at 128 registers/thread: 64 KB).  Lane u
+// of a warp owns slots {d*U + u}: step g loads group g (U consecutive bucket entries of the
+// warp's current chunk) into buffer g % depth and stores group g - (depth - 1) from its
+// buffer, so depth - 1 groups of loads overlap every store.  Chunks come from the same
+// atomic cursor as the LDG path (padding by every SM whose own group drained).
+__device__ __forceinline__ void local_bulk_copy(const GatherParams &p, uint8_t *wsmem, uint64_t *bars,
+                                                uint32_t *oidx, int lane) {
+  const uint32_t R = p.row_bytes;
+  const int slots = min(kBulkMaxSlots, (int)(kBulkWarpBytes / R));
+  const int U = min(kRowsInFlight, slots / 2);
+  const int depth = slots / U;
+  const uint32_t cnt = p.ctrl->counts[p.local_src];
+  const uint64_t *b = p.buckets + (uint64_t)p.local_src * p.bucket_cap;
+  const uint8_t *base = p.base[p.local_src];
+  if (lane < U)
+    for (int d = 0; d < depth; ++d) mbar_init(&bars[d * U + lane], 1);
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  __syncwarp();
+  const uint64_t out_policy = l2_evict_first_policy();
+  uint32_t phase = 0;     // bit d: parity of buffer d's barrier for this lane
+  uint32_t g = 0;         // groups issued by this warp
+  uint32_t valid = 0;     // bit d: this lane loaded a row into buffer d, store pending
+  auto store_group = [&](uint32_t h) {  // wait for group h's row and send it to out
+    const int d = (int)(h % (uint32_t)depth);
+    if (lane < U && (valid >> d & 1u)) {
+      const int slot = d * U + lane;
+      mbar_wait(&bars[slot], (phase >> d) & 1u);
+      phase ^= 1u << d;
+      bulk_s2g(p.out + (uint64_t)oidx[slot] * R, wsmem + (uint32_t)slot * R, R, out_policy);
+      valid &= ~(1u << d);
+    }
+  };
+  uint32_t next = 0;
+  if (lane == 0) next = atomicAdd(&p.ctrl->local_cursor, (uint32_t)kLocalChunk);
+  next = __shfl_sync(kFullMask, next, 0);
+  while (next < cnt) {
+    const uint32_t c0 = next, c1 = min(cnt, c0 + (uint32_t)kLocalChunk);
+    if (lane == 0) next = atomicAdd(&p.ctrl->local_cursor, (uint32_t)kLocalChunk);  // prefetch claim
+    next = __shfl_sync(kFullMask, next, 0);
+    for (uint32_t e0 = c0; e0 < c1; e0 += (uint32_t)U, ++g) {
+      const int d = (int)(g % (uint32_t)depth);
+      if (lane < U && e0 + lane < c1) {
+        const uint64_t ent = b[e0 + lane];
+        const int slot = d * U + lane;
+        bulk_wait_read_all();  // this slot's previous store has left shared memory
+        oidx[slot] = (uint32_t)(ent & 0xFFFFFFFFull);
+        mbar_expect_tx(&bars[slot], R);
+        bulk_g2s(wsmem + (uint32_t)slot * R, base + (ent >> 32) * (uint64_t)R, R, &bars[slot]);
+        valid |= 1u << d;
+      }
+      if (g + 1 >= (uint32_t)depth) store_group(g + 1 - depth);
+    }
+  }
+  for (uint32_t h = g + 1 > (uint32_t)depth ? g + 1 - depth : 0; h < g; ++h) store_group(h);
+  bulk_wait_all();
+}
+
 // ---------------------------------------------------------------------------- K2
 __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_dyn) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -425,6 +548,7 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
   const uint32_t n_host = p.ctrl->counts[host_src];
   const bool host_dense = p.host_sort && n_host >= p.host_sort_min;
   const uint32_t R = p.row_bytes;
+  bool host_cta = false;  // SM-granular mode: this CTA holds a host role
 
   if (p.warp_dedication) {
     // Warp-granular dedication: on EVERY SM, warps [0, hw) serve the
@@ -457,6 +581,7 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
   int my_src, my_idx, role_ctas;
   if (pos < H) {
     my_src = host_src, my_idx = pos, role_ctas = H;
+    host_cta = true;
   } else if (pos - H < p.n_peers * p.peer_sms) {
     my_src = p.peer_src[(pos - H) / p.peer_sms];
     my_idx = (pos - H) % p.peer_sms, role_ctas = p.peer_sms;
@@ -505,7 +630,17 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
   }
   }
   // local group: dedicated local CTAs start here; others pad once their group drains
-  {
+  // TMA bulk local copies (1 always; 2 = unless the host bucket is dense -- with a
+  // PCIe-bound batch the register path's gentler local burst keeps the host reads faster,
+  // DESIGN.md section 6; 3 = on every CTA without a host role)
+  const bool use_bulk = p.local_bulk == 1 || (p.local_bulk == 2 && !host_dense) ||
+                        (p.local_bulk == 3 && !host_cta);
+  if (use_bulk) {
+    __shared__ __align__(8) uint64_t s_bars[kGatherWarps][kBulkMaxSlots];
+    __shared__ uint32_t s_oidx[kGatherWarps][kBulkMaxSlots];
+    local_bulk_copy(p, reinterpret_cast<uint8_t *>(s_dyn) + kRangeTabBytes + warp * kBulkWarpBytes,
+                    s_bars[warp], s_oidx[warp], lane);
+  } else {
     const uint32_t cnt = p.ctrl->counts[p.local_src];
     const uint64_t *b = p.buckets + (uint64_t)p.local_src * p.bucket_cap;
     const uint8_t *base = p.base[p.local_src];
@@ -542,9 +677,11 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
   __shared__ uint32_t s_base[kMaxSrc];
   constexpr uint32_t kTile = kGatherThreads * kLocateItems;
   const uint32_t ntiles = (lp.n + kTile - 1) / kTile;
+  if (blockIdx.x == 0 && threadIdx.x == 0) gp.ctrl->t_start = globaltimer_ns();
   for (uint32_t t = blockIdx.x; t < ntiles; t += gridDim.x)
     locate_tile<KeyT, kGatherThreads>(lp, t, s_cnt, s_base);
   role_barrier(&gp.ctrl->grid_arrive, gridDim.x);
+  if (blockIdx.x == 0 && threadIdx.x == 0) gp.ctrl->t_located = globaltimer_ns();
   gather_body(gp, s_dyn);
 }
 

@@ -70,6 +70,7 @@ struct ugache_ctx {
   int host_rows = ugk::kRowsInFlight;        // env UGACHE_HOST_ROWS (1, 2, 4, 8)
   int host_walk = 1;                         // UGACHE_OPT_HOST_WALK
   int fused = 2;                             // UGACHE_OPT_FUSED: 0 off, 1 on, 2 auto
+  int local_bulk = 2;                        // UGACHE_OPT_LOCAL_BULK (0 off, 1 on, 2 auto, 3)
   int host_warps = ugk::kHostWarps;  // env UGACHE_HOST_WARPS (A0 calibration knob)
   int stage_host_io = 0;             // env UGACHE_STAGE_HOST_IO=1: stage pinned host I/O too
   std::vector<int> smids;  // sorted %smid values of the device (one per SM)
@@ -79,6 +80,7 @@ struct ugache_ctx {
   // timing
   bool timing = false;
   bool timing_valid = false;
+  bool last_fused = false;  // last timed extract ran K1+K2 as one launch
   cudaEvent_t ev[3] = {};
   int last_launches = 0;
   // message-based baseline: 0 idle, 1 local part done (buckets valid), 2 requests packed
@@ -94,7 +96,7 @@ namespace {
 
 // Dynamic shared memory requested only to guarantee one gather CTA per SM, so that the
 // CTA index -> role mapping is also an SM -> role mapping (P:1620-1627 used MPS for this).
-constexpr size_t kOneCtaPerSmSmem = 120 * 1024;
+constexpr size_t kOneCtaPerSmSmem = ugk::kGatherSmem;
 // UGACHE_OPT_FUSED = auto: batches up to this many keys run K1 + K2 in one launch.
 constexpr uint64_t kFusedAutoMaxKeys = 1u << 20;
 
@@ -368,6 +370,7 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_HOST_SORT_MIN")) ctx->host_sort_min = (uint32_t)atoll(e);
   if (const char *e = getenv("UGACHE_HOST_DYNAMIC")) ctx->host_dynamic = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_HOST_ROWS")) ctx->host_rows = atoi(e);
+  if (const char *e = getenv("UGACHE_LOCAL_BULK")) ctx->local_bulk = std::max(0, std::min(3, atoi(e)));
   if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_HOST_WARPS")) ctx->host_warps = std::max(1, std::min(ugk::kGatherWarps, atoi(e)));
   for (int i = 0; i < 3; ++i) UG_CUDA(ctx, cudaEventCreate(&ctx->ev[i]));
@@ -759,6 +762,10 @@ ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value) 
       if (value < 0 || value > 2) return UGACHE_EINVAL;
       ctx->fused = (int)value;
       return UGACHE_OK;
+    case UGACHE_OPT_LOCAL_BULK:
+      if (value < 0 || value > 3) return UGACHE_EINVAL;
+      ctx->local_bulk = (int)value;
+      return UGACHE_OK;
     case UGACHE_OPT_DEDICATION:
       if (value != UGACHE_DEDICATE_SMS && value != UGACHE_DEDICATE_WARPS) return UGACHE_EINVAL;
       ctx->warp_dedication = value == UGACHE_DEDICATE_WARPS;
@@ -878,6 +885,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     gp.keys_u32 = key_type == UGACHE_KEY_U32;
     gp.host_walk = ctx->host_walk;
     gp.host_warps = ctx->host_warps;
+    gp.local_bulk = R <= ugk::kBulkWarpBytes / 2 ? ctx->local_bulk : 0;
     int grid = 0;
     build_roles(ctx, &gp, &grid);
     if (msg_local) {  // message baseline: no SM reads a peer; the peer buckets stay for msg_*
@@ -897,6 +905,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
       UG_CUDA(ctx, cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(ugk::kGatherThreads), kargs,
                                                kOneCtaPerSmSmem, s));
       ctx->last_launches = 1;
+      ctx->last_fused = true;
     } else {
       const unsigned lgrid = (unsigned)((n + ugk::kLocateTile - 1) / ugk::kLocateTile);
       if (ctx->timing) UG_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
@@ -910,6 +919,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
       UG_CUDA(ctx, cudaLaunchCooperativeKernel((const void *)ugk::factored_gather_kernel, dim3(grid),
                                                dim3(ugk::kGatherThreads), kargs, kOneCtaPerSmSmem, s));
       ctx->last_launches = 2;
+      ctx->last_fused = false;
     }
   }
   if (ctx->timing) {
@@ -1067,6 +1077,14 @@ ugache_status ugache_last_batch_timing(ugache_ctx *ctx, float *ms_locate, float 
   float a = 0, b = 0;
   UG_CUDA(ctx, cudaEventElapsedTime(&a, ctx->ev[0], ctx->ev[1]));
   UG_CUDA(ctx, cudaEventElapsedTime(&b, ctx->ev[1], ctx->ev[2]));
+  if (ctx->last_fused && ctx->mode == UGACHE_MODE_FACTORED) {
+    // one launch: split it at the grid barrier with the kernel's own %globaltimer stamps
+    ugk::Ctrl c;
+    UG_CUDA(ctx, cudaMemcpy(&c, ctx->d_ctrl, sizeof(c), cudaMemcpyDeviceToHost));
+    const float loc = c.t_located > c.t_start ? (float)((c.t_located - c.t_start) * 1e-6) : 0.f;
+    a = std::min(loc, b);
+    b -= a;
+  }
   if (ms_locate) *ms_locate = a;
   if (ms_gather) *ms_gather = b;
   return UGACHE_OK;

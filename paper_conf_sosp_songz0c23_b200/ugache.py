@@ -192,6 +192,11 @@ class UGache:
         if peer_warps:
             self.set_option(_abi.OPT_WARP_PEER, peer_warps)
 
+    def set_local_bulk(self, mode):
+        """Local rows by TMA bulk copies: False/0 never, True/1 always, 2 auto (default:
+        unless the host bucket is dense), 3 on CTAs without a host role."""
+        self.set_option(_abi.OPT_LOCAL_BULK, int(mode))
+
     def set_fused(self, mode):
         """'off' (two launches), 'on' (one cooperative launch) or 'auto'."""
         self.set_option(_abi.OPT_FUSED, {"off": 0, "on": 1, "auto": 2}[mode])

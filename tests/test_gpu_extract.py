@@ -148,13 +148,17 @@ def test_all_host_and_all_local(torch_cuda, C):
         c.close()
 
 
-@pytest.mark.parametrize("R", [16, 48, 1536, 2064])
-def test_row_sizes(torch_cuda, R):
+@pytest.mark.parametrize("R", [16, 48, 512, 1536, 2064, 6144, 8192])
+@pytest.mark.parametrize("bulk", [True, False])
+def test_row_sizes(torch_cuda, R, bulk):
+    """Row sizes from one 16-B vector to 8 KB, local rows by TMA bulk copies (R <= 6 KB)
+    or through registers; several chunk and group boundaries per warp."""
     N = 20_000
     h = (synth.zipf_pmf(N, 1.2) * 1e4).astype(np.float32)[np.random.default_rng(R).permutation(N)]
     t, group = make_group(torch_cuda, N, R, 1500, 2, h)
     keys = np.random.default_rng(2).integers(0, N, 7777)
     for c in group:
+        c.set_local_bulk(bulk)
         check_batch(torch_cuda, c, t, keys, N, R, 2)
     for c in group:
         c.close()
@@ -493,6 +497,7 @@ def test_fused_and_split_launch_parity(torch_cuda, fused, G, C, n):
     keys = np.random.default_rng(42).integers(-2, N + 2, n)
     for g, c in enumerate(group):
         c.set_fused(fused)
+        c.set_local_bulk(g % 2 == 0)
         for kd in (np.int64, np.uint32):
             check_batch(torch_cuda, c, t, np.abs(keys) if kd == np.uint32 else keys, N, R, G, key_dtype=kd)
             assert c.last_launch_count() == (1 if fused == "on" else 2)
