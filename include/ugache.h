@@ -287,9 +287,15 @@ typedef enum {
   UGACHE_OPT_WARP_PEER = 5,
   UGACHE_OPT_HOST_WALK = 6,
   UGACHE_OPT_FUSED = 7,
-  UGACHE_OPT_LOCAL_BULK = 8
+  UGACHE_OPT_LOCAL_BULK = 8,
+  UGACHE_OPT_EARLY_WALK = 9
 } ugache_option;
-/* UGACHE_OPT_LOCAL_BULK: local rows (A4) move HBM -> shared -> HBM as TMA cp.async.bulk
+/* UGACHE_OPT_EARLY_WALK (default 0): 1 = in the fused launch, CTAs left without a locate
+ *   tile start the input-order host walk at once, so host rows overlap the locate phase;
+ *   the ordered host path then skips the walked keys.  Needs HOST_WALK and HOST_ORDERING on
+ *   and SM-granular dedication.  Off by default: measured on B200, concurrent host reads
+ *   stretch the locate phase 2-10x.
+ * UGACHE_OPT_LOCAL_BULK: local rows (A4) move HBM -> shared -> HBM as TMA cp.async.bulk
  *   copies (no registers per row, ~196 KB in flight per SM) instead of LDG.128 / STG.128
  *   through registers.  0 = never, 1 = always, 2 (default) = unless the host bucket is
  *   dense enough for range-ordered reads (a PCIe-bound batch, where the register path's

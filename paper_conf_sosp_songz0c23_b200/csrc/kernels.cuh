@@ -44,6 +44,7 @@ struct Ctrl {
   uint32_t host_arrive[2];  // intra-role barriers of the host CTAs
   uint32_t host_cursor;     // dynamic cursor over the range-ordered host bucket
   uint32_t grid_arrive;     // grid barrier of the fused locate+gather kernel
+  uint32_t walk_cursor;     // input-order host walk: next key index to claim
   unsigned long long t_start;    // fused kernel: %globaltimer at CTA 0's start (ns)
   unsigned long long t_located;  // fused kernel: %globaltimer when CTA 0 leaves the grid barrier
 };
@@ -118,6 +119,7 @@ struct GatherParams {
   uint32_t n_keys;
   int32_t keys_u32;                // key type: 0 = int64, 1 = uint32
   int32_t host_walk;               // 1 = sparse host buckets use the input-order walk
+  int32_t early_walk;              // fused kernel: CTAs without a locate tile walk for host rows
   int32_t local_bulk;              // local rows by TMA bulk copies: 0 never, 1 always, 2 unless
                                    // the host bucket is dense, 3 on CTAs without a host role
 };
@@ -223,6 +225,7 @@ __device__ __forceinline__ void finish_launch(Ctrl *ctrl, int num_src) {
       c->host_arrive[1] = 0;
       c->host_cursor = 0;
       c->grid_arrive = 0;
+      c->walk_cursor = 0;
       __threadfence();
       c->done = 0;
     }
@@ -318,6 +321,19 @@ __device__ __forceinline__ void role_barrier(uint32_t *ctr, uint32_t n) {
   __syncthreads();
 }
 
+// Wait (without arriving) until n CTAs have arrived at a role_barrier counter.
+__device__ __forceinline__ void role_wait(const uint32_t *ctr, uint32_t n) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t v;
+    do {
+      asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+      if (v < n) __nanosleep(64);
+    } while (v < n);
+  }
+  __syncthreads();
+}
+
 // Exclusive scan of src[0..n) (global) into dst[0..n) (shared); n <= kMaxRanges.
 __device__ __forceinline__ void block_exclusive_scan(const uint32_t *src, uint32_t *dst, uint32_t n) {
   __shared__ uint32_t s_warp[32];
@@ -371,22 +387,29 @@ __device__ __forceinline__ void host_copy_ordered(const GatherParams &p, uint32_
 }
 
 // Range ordering of the host bucket into p.host_sorted: histogram -> barrier -> scan ->
-// scatter -> barrier.  CTAs h = 0..H-1 cooperate with all their threads.
-__device__ __forceinline__ void host_order(const GatherParams &p, const uint64_t *b,
-                                           uint32_t cnt, int h, int H, uint32_t *s_tab) {
+// scatter -> barrier.  CTAs h = 0..H-1 cooperate with all their threads.  Entries whose key
+// index is below `walked` were already copied by the input-order walk (fused kernel, before
+// its grid barrier) and are dropped.  Returns the number of ordered entries.
+__device__ __forceinline__ uint32_t host_order(const GatherParams &p, const uint64_t *b,
+                                               uint32_t cnt, int h, int H, uint32_t *s_tab,
+                                               uint32_t walked) {
   const int tid = threadIdx.x;
   const uint32_t lo = (uint32_t)((uint64_t)cnt * h / H), hi = (uint32_t)((uint64_t)cnt * (h + 1) / H);
   for (uint32_t i = tid; i < p.n_ranges; i += blockDim.x) s_tab[i] = 0;
   __syncthreads();
-  for (uint32_t e = lo + tid; e < hi; e += blockDim.x)
-    atomicAdd(&s_tab[(uint32_t)(b[e] >> 32) >> p.range_shift], 1u);
+  for (uint32_t e = lo + tid; e < hi; e += blockDim.x) {
+    const uint64_t ent = b[e];
+    if ((uint32_t)ent >= walked) atomicAdd(&s_tab[(uint32_t)(ent >> 32) >> p.range_shift], 1u);
+  }
   __syncthreads();
   for (uint32_t i = tid; i < p.n_ranges; i += blockDim.x)
     if (s_tab[i]) atomicAdd(&p.range_count[i], s_tab[i]);
   role_barrier(&p.ctrl->host_arrive[0], (uint32_t)H);
   block_exclusive_scan(p.range_count, s_tab, p.n_ranges);
+  const uint32_t total = s_tab[p.n_ranges - 1] + p.range_count[p.n_ranges - 1];
   for (uint32_t e = lo + tid; e < hi; e += blockDim.x) {
     const uint64_t ent = b[e];
+    if ((uint32_t)ent < walked) continue;
     const uint32_t r = (uint32_t)(ent >> 32) >> p.range_shift;
     p.host_sorted[s_tab[r] + atomicAdd(&p.range_cursor[r], 1u)] = ent;
   }
@@ -398,13 +421,59 @@ __device__ __forceinline__ void host_order(const GatherParams &p, const uint64_t
       p.range_cursor[i] = 0;
     }
   }
+  return total;
+}
+
+// Input-order host walk (sparse host buckets, and the fused kernel's early walk): warps
+// claim kWalkChunk consecutive keys from a shared cursor, re-read their location entries and
+// copy the host rows among them.  Stops when the keys run out or, with stop != nullptr, once
+// *stop reaches stop_at (checked between claims, so every claimed chunk completes).
+constexpr uint32_t kWalkChunk = 64;
+__device__ __forceinline__ void host_walk_copy(const GatherParams &p, int warp, int lane,
+                                          const uint32_t *stop, uint32_t stop_at) {
+  __shared__ uint64_t s_ent[kGatherWarps][kRowsInFlight];
+  const int host_src = p.num_src - 1;
+  while (true) {
+    uint32_t c0 = 0;
+    if (lane == 0) {
+      bool go = true;
+      if (stop) {
+        uint32_t v;
+        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(stop) : "memory");
+        go = v < stop_at;
+      }
+      c0 = go ? atomicAdd(&p.ctrl->walk_cursor, kWalkChunk) : 0xFFFFFFFFu;
+    }
+    c0 = __shfl_sync(kFullMask, c0, 0);
+    if (c0 >= p.n_keys) return;
+    const uint32_t c1 = min(p.n_keys, c0 + kWalkChunk);
+    for (uint32_t e0 = c0; e0 < c1; e0 += kRowsInFlight) {
+      const int nv = (int)min((uint32_t)kRowsInFlight, c1 - e0);
+      uint64_t ent = ~0ull;
+      if (lane < nv) {
+        const uint64_t i = e0 + lane;
+        const int64_t k = p.keys_u32 ? (int64_t)static_cast<const uint32_t *>(p.keys)[i]
+                                     : static_cast<const int64_t *>(p.keys)[i];
+        if (k >= 0 && (uint64_t)k < p.num_rows) {
+          const uint64_t l = ld_nc_u64(p.loc + k);
+          if ((int)(l >> UGACHE_LOC_SRC_SHIFT) == host_src) ent = ((l & UGACHE_LOC_ROW_MASK) << 32) | i;
+        }
+      }
+      const uint32_t m = __ballot_sync(kFullMask, ent != ~0ull);
+      if (ent != ~0ull) s_ent[warp][__popc(m & lanemask_lt())] = ent;  // compact to lanes 0..
+      __syncwarp();
+      if (m) copy_rows<kRowsInFlight>(p.base[host_src], p.out, p.row_bytes, s_ent[warp], __popc(m), lane);
+      __syncwarp();
+    }
+  }
 }
 
 // Host role (SM-granular dedication) with range ordering: the host CTAs order the bucket,
 // then `host_warps` warps of each copy rows in order; the other warps pad local work.
 __device__ __forceinline__ void host_role_sorted(const GatherParams &p, const uint64_t *b,
-                                                 uint32_t cnt, int h, int H, uint32_t *s_tab) {
-  host_order(p, b, cnt, h, H, s_tab);
+                                                 uint32_t cnt, int h, int H, uint32_t *s_tab,
+                                                 uint32_t walked) {
+  cnt = host_order(p, b, cnt, h, H, s_tab, walked);
   if ((int)(threadIdx.x >> 5) >= p.host_warps) return;  // window control
   host_copy_ordered<kRowsInFlight>(p, cnt, threadIdx.x & 31);
 }
@@ -548,6 +617,8 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
   const uint32_t n_host = p.ctrl->counts[host_src];
   const bool host_dense = p.host_sort && n_host >= p.host_sort_min;
   const uint32_t R = p.row_bytes;
+  // keys [0, walked) were walked for host rows before the fused kernel's grid barrier
+  const uint32_t walked = min(*(volatile const uint32_t *)&p.ctrl->walk_cursor, p.n_keys);
   bool host_cta = false;  // SM-granular mode: this CTA holds a host role
 
   if (p.warp_dedication) {
@@ -557,9 +628,9 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
     // and no SM idles behind a slow link.
     const int S = p.num_sms, hw = p.host_warps, pw = p.peer_warps;
     const uint64_t *bh = p.buckets + (uint64_t)host_src * p.bucket_cap;
-    if (host_dense) host_order(p, bh, n_host, pos, S, s_dyn);
+    const uint32_t n_ord = host_dense ? host_order(p, bh, n_host, pos, S, s_dyn, 0) : 0;
     if (warp < hw) {
-      if (host_dense) host_copy_ordered<kRowsInFlight>(p, n_host, lane);
+      if (host_dense) host_copy_ordered<kRowsInFlight>(p, n_ord, lane);
       else stride_copy(p, bh, n_host, p.base[host_src], (uint32_t)(pos * hw + warp), (uint32_t)(S * hw), lane,
                        p.host_rows);
     } else if (warp < hw + p.n_peers * pw) {
@@ -591,34 +662,14 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
 
   if (my_src == host_src && host_walk) {
     // Sparse host bucket: the host SMs walk the batch's keys in input order (re-reading
-    // their location entries) and copy the host rows they meet.  Measured on the B200 box,
-    // sparse cold host rows are read ~1.6x faster in this paced input order than from the
-    // dense host bucket, whose rows would all be requested at once.
-    __shared__ uint64_t s_ent[kGatherWarps][kRowsInFlight];
-    const uint32_t W = (uint32_t)role_ctas * kGatherWarps;
-    for (uint32_t e0 = ((uint32_t)my_idx * kGatherWarps + warp) * kRowsInFlight; e0 < p.n_keys;
-         e0 += W * kRowsInFlight) {
-      const int nv = (int)min((uint32_t)kRowsInFlight, p.n_keys - e0);
-      uint64_t ent = ~0ull;
-      if (lane < nv) {
-        const uint64_t i = e0 + lane;
-        const int64_t k = p.keys_u32 ? (int64_t)static_cast<const uint32_t *>(p.keys)[i]
-                                     : static_cast<const int64_t *>(p.keys)[i];
-        if (k >= 0 && (uint64_t)k < p.num_rows) {
-          const uint64_t l = ld_nc_u64(p.loc + k);
-          if ((int)(l >> UGACHE_LOC_SRC_SHIFT) == host_src)
-            ent = ((l & UGACHE_LOC_ROW_MASK) << 32) | i;
-        }
-      }
-      const uint32_t m = __ballot_sync(kFullMask, ent != ~0ull);
-      if (ent != ~0ull) s_ent[warp][__popc(m & lanemask_lt())] = ent;  // compact to lanes 0..
-      __syncwarp();
-      if (m) copy_rows<kRowsInFlight>(p.base[host_src], p.out, R, s_ent[warp], __popc(m), lane);
-      __syncwarp();
-    }
+    // their location entries) and copy the host rows they meet, continuing where the fused
+    // kernel's early walk stopped.  Measured on the B200 box, sparse cold host rows are read
+    // ~1.6x faster in this paced input order than from the dense host bucket, whose rows
+    // would all be requested at once.
+    host_walk_copy(p, warp, lane, nullptr, 0);
   } else if (my_src == host_src && host_dense) {
     host_role_sorted(p, p.buckets + (uint64_t)host_src * p.bucket_cap, n_host, my_idx, role_ctas,
-                     s_dyn);
+                     s_dyn, walked);
   } else if (my_src != p.local_src) {
     // dedicated non-local extraction: static warp striding over this source's bucket
     const uint32_t cnt = p.ctrl->counts[my_src];
@@ -678,10 +729,27 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
   constexpr uint32_t kTile = kGatherThreads * kLocateItems;
   const uint32_t ntiles = (lp.n + kTile - 1) / kTile;
   if (blockIdx.x == 0 && threadIdx.x == 0) gp.ctrl->t_start = globaltimer_ns();
-  for (uint32_t t = blockIdx.x; t < ntiles; t += gridDim.x)
+  // Tiles go to CTAs in chip-spreading order; CTAs left without a tile start the input-order
+  // host walk at once (the host rows of a sparse batch then overlap the locate phase, as in
+  // the unfactored kernel) until every tile is located.  Keys walked here are skipped by the
+  // ordered host path after the barrier (host_order's `walked`).
+  // Walkers never arrive at the barrier (it counts the locating CTAs only), so a walker
+  // finishing its last chunk delays nobody; claimed chunks are always completed by their
+  // claimer, so skipping [0, walked) in the ordered path stays exact.
+  uint32_t smid;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+  const uint32_t pos = smid < (uint32_t)kMaxSmId ? gp.sm_pos[smid] : blockIdx.x;
+  const bool walker = gp.early_walk && pos >= ntiles;
+  const uint32_t arrivals = gp.early_walk ? min(gridDim.x, ntiles) : gridDim.x;
+  for (uint32_t t = pos; t < ntiles; t += gridDim.x)
     locate_tile<KeyT, kGatherThreads>(lp, t, s_cnt, s_base);
-  role_barrier(&gp.ctrl->grid_arrive, gridDim.x);
-  if (blockIdx.x == 0 && threadIdx.x == 0) gp.ctrl->t_located = globaltimer_ns();
+  if (walker) {
+    host_walk_copy(gp, threadIdx.x >> 5, threadIdx.x & 31, &gp.ctrl->grid_arrive, arrivals);
+    role_wait(&gp.ctrl->grid_arrive, arrivals);
+  } else {
+    role_barrier(&gp.ctrl->grid_arrive, arrivals);
+  }
+  if (pos == 0 && threadIdx.x == 0) gp.ctrl->t_located = globaltimer_ns();
   gather_body(gp, s_dyn);
 }
 

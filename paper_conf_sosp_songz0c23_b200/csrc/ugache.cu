@@ -70,6 +70,7 @@ struct ugache_ctx {
   int host_rows = ugk::kRowsInFlight;        // env UGACHE_HOST_ROWS (1, 2, 4, 8)
   int host_walk = 1;                         // UGACHE_OPT_HOST_WALK
   int fused = 2;                             // UGACHE_OPT_FUSED: 0 off, 1 on, 2 auto
+  int early_walk = 0;                        // UGACHE_OPT_EARLY_WALK (env UGACHE_EARLY_WALK)
   int local_bulk = 2;                        // UGACHE_OPT_LOCAL_BULK (0 off, 1 on, 2 auto, 3)
   int host_warps = ugk::kHostWarps;  // env UGACHE_HOST_WARPS (A0 calibration knob)
   int stage_host_io = 0;             // env UGACHE_STAGE_HOST_IO=1: stage pinned host I/O too
@@ -370,6 +371,7 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_HOST_SORT_MIN")) ctx->host_sort_min = (uint32_t)atoll(e);
   if (const char *e = getenv("UGACHE_HOST_DYNAMIC")) ctx->host_dynamic = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_HOST_ROWS")) ctx->host_rows = atoi(e);
+  if (const char *e = getenv("UGACHE_EARLY_WALK")) ctx->early_walk = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_LOCAL_BULK")) ctx->local_bulk = std::max(0, std::min(3, atoi(e)));
   if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_HOST_WARPS")) ctx->host_warps = std::max(1, std::min(ugk::kGatherWarps, atoi(e)));
@@ -762,6 +764,10 @@ ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value) 
       if (value < 0 || value > 2) return UGACHE_EINVAL;
       ctx->fused = (int)value;
       return UGACHE_OK;
+    case UGACHE_OPT_EARLY_WALK:
+      if (value < 0 || value > 1) return UGACHE_EINVAL;
+      ctx->early_walk = (int)value;
+      return UGACHE_OK;
     case UGACHE_OPT_LOCAL_BULK:
       if (value < 0 || value > 3) return UGACHE_EINVAL;
       ctx->local_bulk = (int)value;
@@ -886,6 +892,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     gp.host_walk = ctx->host_walk;
     gp.host_warps = ctx->host_warps;
     gp.local_bulk = R <= ugk::kBulkWarpBytes / 2 ? ctx->local_bulk : 0;
+    gp.early_walk = ctx->early_walk && ctx->host_walk && ctx->host_sort && !ctx->warp_dedication && !msg_local;
     int grid = 0;
     build_roles(ctx, &gp, &grid);
     if (msg_local) {  // message baseline: no SM reads a peer; the peer buckets stay for msg_*

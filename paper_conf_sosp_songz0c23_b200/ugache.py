@@ -192,6 +192,10 @@ class UGache:
         if peer_warps:
             self.set_option(_abi.OPT_WARP_PEER, peer_warps)
 
+    def set_early_walk(self, on: bool):
+        """Fused launch: CTAs without a locate tile walk for host rows before the barrier."""
+        self.set_option(_abi.OPT_EARLY_WALK, int(on))
+
     def set_local_bulk(self, mode):
         """Local rows by TMA bulk copies: False/0 never, True/1 always, 2 auto (default:
         unless the host bucket is dense), 3 on CTAs without a host role."""

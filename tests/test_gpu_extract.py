@@ -540,3 +540,27 @@ def test_message_based_baseline_parity(torch_cuda, G, policy, fused):
         message._scatter(group[0], outs[0], outs[0], None)
     for c in group:
         c.close()
+
+
+@pytest.mark.parametrize("early", [True, False])
+@pytest.mark.parametrize("G,C,n", [(1, 2000, 30_000), (1, 2000, 700_000), (2, 20_000, 120_000),
+                                   (4, 60_000, 8_193)])
+def test_early_host_walk_parity(torch_cuda, early, G, C, n):
+    """Fused launch with CTAs that have no locate tile walking for host rows before the grid
+    barrier: dense host buckets (the ordered path must skip the walked prefix), sparse ones
+    (the post-barrier walk continues from the shared cursor), and batches with more tiles
+    than CTAs (no early walkers)."""
+    N, R = 400_000, 512
+    h = (synth.zipf_pmf(N, 1.1) * 1e5).astype(np.float32)[np.random.default_rng(43).permutation(N)]
+    t, group = make_group(torch_cuda, N, R, C, G, h)
+    rng = np.random.default_rng(44)
+    for g, c in enumerate(group):
+        c.set_fused("on")
+        c.set_early_walk(early)
+        for b in range(3):  # repeated launches: the walk cursor is re-armed by the kernel
+            keys = rng.integers(0, N, n)
+            keys[:: 997] = N + 1
+            per = check_batch(torch_cuda, c, t, keys, N, R, G)
+            assert per[G] > 0
+    for c in group:
+        c.close()
