@@ -49,6 +49,10 @@ def parse():
     ap.add_argument("--cache-ratio", type=float, default=None)
     ap.add_argument("--policy", default="ugache")
     ap.add_argument("--mode", default="factored", choices=["factored", "random"])
+    ap.add_argument("--stream", default="auto", choices=["off", "on", "auto"],
+                    help="single-pass extraction (UGACHE_OPT_STREAM)")
+    ap.add_argument("--inline", default="host", choices=["host", "none", "all"],
+                    help="single pass: sources copied by the locating warps (UGACHE_OPT_INLINE)")
     ap.add_argument("--host-sms", type=int, default=0)
     ap.add_argument("--peer-sms", type=int, default=0)
     ap.add_argument("--batches", type=int, default=4, help="distinct batches cycled per rank")
@@ -208,11 +212,13 @@ def config_dict(args, wl, ws):
             "payload": f"{wl.row_bytes // (2 if wl.dtype == 'f16' else 4)} x {wl.dtype}",
             "keys_per_batch_per_gpu": wl.keys_per_batch, "batch_kind": wl.batch_kind,
             "alpha": wl.alpha, "cache_ratio": args.cache_ratio if args.cache_ratio is not None
-            else wl.cache_ratio, "policy": args.policy, "mode": args.mode,
+            else wl.cache_ratio, "policy": args.policy, "mode": args.mode, "stream": args.stream, "inline": args.inline,
             "host_tier": bool(getattr(args, "host_tier", False)),
             "parallelism": f"dp{ws}",
             "l2": "256 MiB L2-flush write between timed steps (outside the events); per-step "
-                  "output > L2"}
+                  "output > L2",
+            "launch_gap": "a ~50 us device spin precedes each timed step (outside the events) so "
+                          "the host has enqueued the step before its start event fires"}
 
 
 def main():
@@ -285,6 +291,8 @@ def main():
     log(f"fill in {time.time() - t0:.2f}s")
     if args.mode == "random":
         cache.set_mode("random")
+    cache.set_stream(args.stream)
+    cache.set_inline(host=args.inline != "none", peers=args.inline == "all")
 
     batches = make_batches(wl, rank, max(1, min(args.batches, args.steps + args.warmup)))
     n = len(batches[0])
@@ -297,6 +305,10 @@ def main():
     def step(i, timed):
         with torch.cuda.stream(stream):
             flush.fill_(i & 0xFF)  # evict L2 between steps (outside the events)
+            # ~50 us of device spin, also outside the events: the host enqueues the step
+            # while the GPU is busy, so the events time the step's device work, not the
+            # Python/launch latency (that is in the e2e number)
+            torch.cuda._sleep(100_000)
         if timed:
             s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             s.record(stream)

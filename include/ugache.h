@@ -288,8 +288,29 @@ typedef enum {
   UGACHE_OPT_HOST_WALK = 6,
   UGACHE_OPT_FUSED = 7,
   UGACHE_OPT_LOCAL_BULK = 8,
-  UGACHE_OPT_EARLY_WALK = 9
+  UGACHE_OPT_EARLY_WALK = 9,
+  UGACHE_OPT_STREAM = 10,
+  UGACHE_OPT_INLINE = 11
 } ugache_option;
+/* UGACHE_OPT_STREAM: single-pass extraction (K3, its own cooperative kernel).  Warps take
+ *   64-key chunks (a static schedule: warp w takes chunks w, w + W, ...), locate them (A1)
+ *   and copy local rows at once (A4: local extraction tolerates every core);
+ *   rows of a queued source go to that source's queue, drained only by the SMs dedicated to
+ *   it (A2/A3), which locate chunks themselves while their queue is empty.
+ *   Rows move through per-lane TMA shared-memory slots (cp.async.bulk in and out, up to
+ *   12 KB in flight per warp).  No grid barrier and no bucket round trip for local rows.
+ *   0 = off (locate | grid barrier | factored gather); 1 = always; 2 (default) = for rows of
+ *   at most 1 KB, unless the last launch on this ctx had a host bucket dense enough for
+ *   range-ordered reads (scaled to this batch's size; the kernel mirrors its counts to
+ *   pinned host memory, so the choice needs no synchronisation).  Ignored with
+ *   UGACHE_DEDICATE_WARPS and on the message path.  Timing reports the whole launch as
+ *   the gather phase (locate = 0).
+ * UGACHE_OPT_INLINE: bit mask of the sources whose rows the locating warp copies itself in
+ *   single-pass mode instead of queueing them for dedicated SMs: UGACHE_INLINE_HOST (default)
+ *   -- on the B200 box sparse host rows are latency/translation-bound,
+ *   so spreading them over every warp beats a bounded set of dedicated warps -- and
+ *   UGACHE_INLINE_PEERS (ablation: no peer dedication). */
+enum { UGACHE_INLINE_HOST = 1, UGACHE_INLINE_PEERS = 2 };
 /* UGACHE_OPT_EARLY_WALK (default 0): 1 = in the fused launch, CTAs left without a locate
  *   tile start the input-order host walk at once, so host rows overlap the locate phase;
  *   the ordered host path then skips the walked keys.  Needs HOST_WALK and HOST_ORDERING on

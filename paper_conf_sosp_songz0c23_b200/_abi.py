@@ -26,7 +26,8 @@ KEY_I64, KEY_U32 = 0, 1
 MODE_FACTORED, MODE_RANDOM_DISPATCH = 0, 1
 OPT_HOST_ORDERING, OPT_STAGE_HOST_IO, OPT_HOST_WARPS = 0, 1, 2
 OPT_DEDICATION, OPT_WARP_HOST, OPT_WARP_PEER, OPT_HOST_WALK, OPT_FUSED = 3, 4, 5, 6, 7
-OPT_LOCAL_BULK, OPT_EARLY_WALK = 8, 9
+OPT_LOCAL_BULK, OPT_EARLY_WALK, OPT_STREAM, OPT_INLINE = 8, 9, 10, 11
+INLINE_HOST, INLINE_PEERS = 1, 2
 DEDICATE_SMS, DEDICATE_WARPS = 0, 1
 FLAG_HOST_TIER = 1
 

@@ -47,6 +47,15 @@ struct Ctrl {
   uint32_t walk_cursor;     // input-order host walk: next key index to claim
   unsigned long long t_start;    // fused kernel: %globaltimer at CTA 0's start (ns)
   unsigned long long t_located;  // fused kernel: %globaltimer when CTA 0 leaves the grid barrier
+  // single-pass (streaming) extraction
+  uint32_t qhead[kMaxSrc];  // consumer cursor of each source's queue
+  uint32_t chunk_cursor;    // next key chunk to locate
+  uint32_t keys_done;       // keys whose chunk is fully located (queued or copied)
+  uint32_t stat_n;          // keys of the last launch (auto mode: previous batch's host density)
+  uint32_t last_stream;     // 1 = the last launch ran the single-pass path
+  // pinned, device-mapped host words {n, host count, launches} written by the last CTA of
+  // every launch: the host picks the next batch's path from them without synchronising
+  volatile uint32_t *host_mirror;
 };
 
 __device__ __forceinline__ unsigned long long globaltimer_ns() {
@@ -122,6 +131,16 @@ struct GatherParams {
   int32_t early_walk;              // fused kernel: CTAs without a locate tile walk for host rows
   int32_t local_bulk;              // local rows by TMA bulk copies: 0 never, 1 always, 2 unless
                                    // the host bucket is dense, 3 on CTAs without a host role
+  // single-pass extraction (fused kernel only; stream_body)
+  int32_t inline_host;             // single pass: host rows copied by the locating warp
+  int32_t inline_peer;             // single pass: peer rows copied by the locating warp (ablation)
+  uint64_t *queues;                // num_src x bucket_cap entries, ~0 between launches
+  int32_t stream_bulk;             // single pass: inline rows through TMA slots (StreamSlots)
+  int32_t stream_k;                // single pass: keys per lane per chunk (1 or 2)
+  int32_t stream_host_last;        // single pass: non-local inline rows after the local ones
+  int32_t stream_host_cap;         // single pass: non-local rows in flight per warp (0 = slots)
+  int32_t stream_static;           // single pass: static chunk schedule instead of the cursor
+  int32_t stream_nap;              // single pass: ns a warp sleeps when all its slots are in flight
 };
 
 struct RandomParams {
@@ -206,7 +225,7 @@ __device__ __forceinline__ bool key_in_range(KeyT k, uint64_t N) {
 }
 
 // Last CTA of a gather launch publishes stats and re-arms the control block.
-__device__ __forceinline__ void finish_launch(Ctrl *ctrl, int num_src) {
+__device__ __forceinline__ void finish_launch(Ctrl *ctrl, int num_src, uint32_t n, uint32_t streamed) {
   __syncthreads();
   if (threadIdx.x == 0) {
     __threadfence();
@@ -217,6 +236,16 @@ __device__ __forceinline__ void finish_launch(Ctrl *ctrl, int num_src) {
       for (int s = 0; s < num_src; ++s) {
         c->stat_counts[s] = c->counts[s];
         c->counts[s] = 0;
+        c->qhead[s] = 0;
+      }
+      c->chunk_cursor = 0;
+      c->keys_done = 0;
+      c->stat_n = n;
+      c->last_stream = streamed;
+      if (c->host_mirror) {
+        c->host_mirror[0] = n;
+        c->host_mirror[1] = c->stat_counts[num_src - 1];
+        c->host_mirror[2] = c->host_mirror[2] + 1;
       }
       c->stat_bad = c->bad;
       c->bad = 0;
@@ -707,13 +736,397 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
                                  lane);
     }
   }
-  finish_launch(p.ctrl, p.num_src);
+  finish_launch(p.ctrl, p.num_src, p.n_keys, 0);
 }
 
 __global__ void __launch_bounds__(kGatherThreads, 1)
     factored_gather_kernel(const GatherParams p) {
   extern __shared__ __align__(16) uint32_t s_dyn[];
   gather_body(p, s_dyn);
+}
+
+// ---------------------------------------------------------------------------- single pass
+// Single-pass extraction (K3, the fused kernel's `stream` path).  The locate of A1 and the
+// copies of A3/A4 overlap instead of meeting at a grid barrier: warps claim 64-key chunks in
+// input order, look their keys up, copy the rows they may copy themselves at once (local
+// rows -- local extraction "can tolerate all GPU cores", P:1096-1103 -- plus inline host /
+// peer rows) and append every other row to its source's queue, which only that source's
+// dedicated SMs drain (A2/A3 core dedication).  Local rows never touch a
+// bucket, so the 16 B/key bucket round trip and the locate->gather barrier disappear.
+// Queues hold (row << 32 | out_idx) entries and are ~0 between launches: a consumer claims
+// an index from the queue's head cursor and waits for the entry to be written; it writes ~0
+// back after reading it.  A source's queue is final once every chunk is located
+// (keys_done == n; reservations precede the increment).
+constexpr int kStreamK = 2;                          // keys per lane per chunk
+constexpr uint32_t kStreamChunk = 32u * kStreamK;    // keys per chunk (one warp)
+constexpr uint32_t kNoClaim = 0xFFFFFFFFu;
+constexpr int kStreamRegRows = 4;                    // rows per step of the register path (R > 6 KB)
+
+__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t *p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t *p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed_u64(uint64_t *p, uint64_t v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// Warp copies up to U rows; lane u < nvalid holds row u's source address and output index.
+template <int U>
+__device__ __forceinline__ void copy_addr_rows(uint8_t *__restrict__ out, uint32_t R, uint64_t src,
+                                               uint32_t oidx, int nvalid, int lane) {
+  uint64_t su[U];
+  uint32_t du[U];
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    su[u] = __shfl_sync(kFullMask, src, u);
+    du[u] = __shfl_sync(kFullMask, oidx, u);
+  }
+  const uint32_t V = R >> 4;
+  for (uint32_t j = lane; j < V; j += 32) {
+    uint4 v[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (u < nvalid) v[u] = ld_nc_v4(reinterpret_cast<const uint8_t *>(su[u]) + (uint64_t)j * 16u);
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (u < nvalid) st_cs_v4(out + (uint64_t)du[u] * R + (uint64_t)j * 16u, v[u]);
+  }
+}
+
+// One chunk: locate its keys, queue the rows of queued sources, copy the rest (non-local
+// inline rows first, so their longer latencies start first).  s_addr / s_idx: this warp's
+// kStreamChunk-entry copy list; s_inl: per-CTA counts of inline rows per source.
+// Asynchronous row slots of one warp (single pass, rows <= 6 KB): lane u < nslots owns one
+// R-byte shared-memory slot and its mbarrier.  A row moves source -> slot by one
+// cp.async.bulk (TMA) and slot -> out by another, both issued by its lane; a lane takes a
+// new row as soon as its slot's row has landed, so a slow row (a cold host read) holds one
+// lane's slot while the other lanes keep streaming local rows: up to nslots rows in flight
+// per warp (12 KB), no registers held per row, and a row's latency is off the warp's
+// critical path.  A slot whose store was issued in this round is reused one round later
+// (its store has usually left shared memory by then, so the reuse wait is short).
+struct StreamSlots {
+  uint8_t *buf;       // this lane's slot
+  uint64_t *bar;      // this lane's mbarrier
+  uint64_t policy;    // L2 policy of the output stores (evict_first)
+  uint32_t oidx;      // output row of the slot's pending row
+  uint32_t phase;     // mbarrier parity
+  uint32_t busy;      // a row is on its way into the slot
+  uint32_t slow;      // ... and it comes from a non-local source
+  int nslots;         // 0: register path (copy_addr_rows)
+  int slow_cap;       // max non-local rows in flight per warp
+  uint32_t nap;       // ns to sleep when every slot is in flight
+
+  __device__ __forceinline__ void init(uint8_t *wbuf, uint64_t *wbars, uint32_t R, int lane, bool on, int cap,
+                                       uint32_t nap_ns) {
+    nap = nap_ns;
+    nslots = on ? min(32, (int)(kBulkWarpBytes / R)) : 0;
+    slow_cap = cap > 0 ? cap : 32;
+    buf = wbuf + (uint32_t)lane * R;
+    bar = wbars + lane;
+    phase = 0, busy = 0, slow = 0, oidx = 0;
+    policy = l2_evict_first_policy();
+    if (lane < nslots) mbar_init(bar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    __syncwarp();
+  }
+  __device__ __forceinline__ bool landed() const {
+    uint32_t done;
+    asm volatile(
+        "{ .reg .pred p; mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(phase)
+        : "memory");
+    return done != 0;
+  }
+  __device__ __forceinline__ void retire(uint8_t *out, uint32_t R) {  // slot -> out
+    phase ^= 1u;
+    busy = 0;
+    slow = 0;
+    bulk_s2g(out + (uint64_t)oidx * R, buf, R, policy);
+  }
+  // Copy list entries [0, nl): free lanes take the next entries in list order; entries
+  // [sb, se) are non-local rows, at most slow_cap of them in flight per warp.
+  __device__ __forceinline__ void feed(const uint64_t *s_addr, const uint32_t *s_idx, uint32_t nl,
+                                       uint32_t sb, uint32_t se, uint8_t *out, uint32_t R, int lane) {
+    uint32_t next = 0;
+    while (next < nl) {
+      const bool free_lane = lane < nslots && !busy;  // free before this round's retirements
+      if (lane < nslots && busy && landed()) retire(out, R);
+      const uint32_t fm = __ballot_sync(kFullMask, free_lane);
+      const uint32_t in_slow = (uint32_t)__popc(__ballot_sync(kFullMask, busy && slow));
+      uint32_t t = min((uint32_t)__popc(fm), nl - next);
+      const uint32_t s0 = max(next, sb), s1 = min(next + t, se);
+      const uint32_t allowed = (uint32_t)slow_cap > in_slow ? (uint32_t)slow_cap - in_slow : 0u;
+      if (s1 > s0 && s1 - s0 > allowed) t = s0 + allowed - next;
+      if (!t) {  // every slot in flight: yield the issue slots to the SM's other warps
+        if (nap) __nanosleep(nap);
+        continue;
+      }
+      const uint32_t e = next + __popc(fm & lanemask_lt());
+      if (free_lane && e < next + t) {
+        bulk_wait_read_all();  // this lane's previous store has left the slot
+        oidx = s_idx[e];
+        slow = e >= sb && e < se;
+        mbar_expect_tx(bar, R);
+        bulk_g2s(buf, reinterpret_cast<const void *>(s_addr[e]), R, bar);
+        busy = 1;
+      }
+      next += t;
+    }
+  }
+  __device__ __forceinline__ void drain(uint8_t *out, uint32_t R, int lane) {
+    if (lane < nslots && busy) {
+      mbar_wait(bar, phase);
+      retire(out, R);
+    }
+    bulk_wait_all();
+    __syncwarp();
+  }
+};
+
+template <typename KeyT>
+__device__ __forceinline__ void stream_keys(const LocateParams &lp, const GatherParams &gp, uint32_t c, int lane,
+                                            KeyT (&k)[kStreamK]) {
+  const KeyT *keys = static_cast<const KeyT *>(lp.keys);
+  const uint32_t K = (uint32_t)gp.stream_k, i0 = c * 32u * K;
+#pragma unroll
+  for (int it = 0; it < kStreamK; ++it) {
+    const uint32_t i = i0 + it * 32 + lane;
+    k[it] = (it < (int)K && i < lp.n) ? keys[i] : (KeyT)0;
+  }
+}
+template <typename KeyT>
+__device__ __forceinline__ void stream_locs(const LocateParams &lp, const GatherParams &gp, uint32_t c, int lane,
+                                            const KeyT (&k)[kStreamK], uint64_t (&e)[kStreamK]) {
+  const uint32_t K = (uint32_t)gp.stream_k, i0 = c * 32u * K;
+#pragma unroll
+  for (int it = 0; it < kStreamK; ++it) {
+    const uint32_t i = i0 + it * 32 + lane;
+    e[it] = (it < (int)K && i < lp.n && key_in_range<KeyT>(k[it], lp.num_rows)) ? ld_nc_u64(lp.loc + (uint64_t)k[it])
+                                                                               : ~0ull;
+  }
+}
+
+// Chunk c whose location entries e[] are loaded (stream_keys + stream_locs).
+template <typename KeyT>
+__device__ __forceinline__ void stream_chunk_located(const LocateParams &lp, const GatherParams &gp, uint32_t c,
+                                                     const uint64_t (&e)[kStreamK], int lane, uint64_t *s_addr,
+                                                     uint32_t *s_idx, uint32_t *s_inl, StreamSlots &sl) {
+  const uint32_t K = (uint32_t)gp.stream_k, chunk = 32u * K;
+  const uint32_t R = gp.row_bytes, n = lp.n, i0 = c * chunk;
+  const int host_src = gp.num_src - 1;
+  int s[kStreamK];
+  uint32_t nbad = 0;
+#pragma unroll
+  for (int it = 0; it < kStreamK; ++it) {
+    const uint32_t i = i0 + it * 32 + lane;
+    s[it] = -1;
+    if (it < (int)K && i < n) {
+      if (e[it] != ~0ull) {
+        s[it] = (int)(e[it] >> UGACHE_LOC_SRC_SHIFT);
+      } else {
+        zero_row(gp.out + (uint64_t)i * R, R);  // out-of-range key
+        ++nbad;
+      }
+    }
+    const int si = s[it];
+    const bool inl = si >= 0 && (si == gp.local_src || (si == host_src ? gp.inline_host : gp.inline_peer));
+    const int qs = (si >= 0 && !inl) ? si : -1;
+    // queued rows: warp-aggregated reservation on the source's queue, then the entry
+    const uint32_t qpeers = __match_any_sync(kFullMask, qs);
+    const int qleader = __ffs(qpeers) - 1;
+    uint32_t b = 0;
+    if (qs >= 0 && lane == qleader) b = atomicAdd(&gp.ctrl->counts[qs], (uint32_t)__popc(qpeers));
+    b = __shfl_sync(kFullMask, b, qleader);
+    if (qs >= 0)
+      st_relaxed_u64(gp.queues + (uint64_t)qs * gp.bucket_cap + b + __popc(qpeers & lanemask_lt()),
+                     ((e[it] & UGACHE_LOC_ROW_MASK) << 32) | (uint64_t)i);
+    // inline rows: per-CTA statistics
+    const int is = inl ? si : -1;
+    const uint32_t ipeers = __match_any_sync(kFullMask, is);
+    if (is >= 0 && lane == __ffs(ipeers) - 1) atomicAdd(&s_inl[is], (uint32_t)__popc(ipeers));
+  }
+  if (nbad) atomicAdd(&gp.ctrl->bad, nbad);
+  // copy list: [inline non-local rows | local rows] (or local first with stream_host_last)
+  uint32_t nl = 0, slow_b = 0, slow_e = 0;
+#pragma unroll
+  for (int pass = 0; pass < 2; ++pass) {
+    const bool slow_pass = (pass == 0) != (gp.stream_host_last != 0);
+    if (slow_pass) slow_b = nl;
+#pragma unroll
+    for (int it = 0; it < kStreamK; ++it) {
+      const int si = s[it];
+      const bool take = si >= 0 && (!slow_pass ? si == gp.local_src
+                                               : si != gp.local_src &&
+                                                     (si == host_src ? gp.inline_host : gp.inline_peer));
+      const uint32_t m = __ballot_sync(kFullMask, take);
+      if (take) {
+        const uint32_t at = nl + __popc(m & lanemask_lt());
+        s_addr[at] = reinterpret_cast<uint64_t>(gp.base[si]) + (e[it] & UGACHE_LOC_ROW_MASK) * (uint64_t)R;
+        s_idx[at] = i0 + it * 32 + lane;
+      }
+      nl += __popc(m);
+    }
+    if (slow_pass) slow_e = nl;
+  }
+  __syncwarp();
+  if (sl.nslots) {
+    sl.feed(s_addr, s_idx, nl, slow_b, slow_e, gp.out, R, lane);
+  } else {
+    for (uint32_t g0 = 0; g0 < nl; g0 += kStreamRegRows) {
+      const int nv = (int)min((uint32_t)kStreamRegRows, nl - g0);
+      const uint64_t a = lane < nv ? s_addr[g0 + lane] : 0ull;
+      const uint32_t o = lane < nv ? s_idx[g0 + lane] : 0u;
+      copy_addr_rows<kStreamRegRows>(gp.out, R, a, o, nv, lane);
+    }
+  }
+  __syncwarp();
+  // this chunk's reservations and queue entries precede its keys_done increment
+  __threadfence();
+  __syncwarp();
+  if (lane == 0) atomicAdd(&gp.ctrl->keys_done, min(chunk, n - i0));
+}
+
+template <typename KeyT>
+__device__ __forceinline__ void stream_chunk(const LocateParams &lp, const GatherParams &gp, uint32_t c, int lane,
+                                             uint64_t *s_addr, uint32_t *s_idx, uint32_t *s_inl, StreamSlots &sl) {
+  KeyT k[kStreamK];
+  uint64_t e[kStreamK];
+  stream_keys<KeyT>(lp, gp, c, lane, k);
+  stream_locs<KeyT>(lp, gp, c, lane, k, e);
+  stream_chunk_located<KeyT>(lp, gp, c, e, lane, s_addr, s_idx, s_inl, sl);
+}
+
+// Dedicated warp: claim up to kRowsInFlight (register path: kStreamRegRows) entries of
+// source s's queue and copy them.
+// Returns false when nothing was reserved beyond the queue head.
+__device__ __forceinline__ bool stream_consume(const GatherParams &gp, int s, uint32_t n, int lane,
+                                               uint64_t *s_addr, uint32_t *s_idx, StreamSlots &sl) {
+  Ctrl *ctrl = gp.ctrl;
+  // Claims never pass the reservation counter (CAS), so every claimed entry is being
+  // written by a producer that does not block: waiting for it cannot deadlock even when
+  // every warp of the grid is a consumer.
+  uint32_t claim = kNoClaim, take = 0;
+  if (lane == 0) {
+    uint32_t h = ld_relaxed_u32(&ctrl->qhead[s]);
+    while (true) {
+      const uint32_t c = ld_relaxed_u32(&ctrl->counts[s]);
+      if (h >= c) break;
+      const uint32_t t = min(sl.nslots ? (uint32_t)kRowsInFlight : (uint32_t)kStreamRegRows, c - h);
+      const uint32_t old = atomicCAS(&ctrl->qhead[s], h, h + t);
+      if (old == h) {
+        claim = h, take = t;
+        break;
+      }
+      h = old;
+    }
+  }
+  claim = __shfl_sync(kFullMask, claim, 0);
+  if (claim == kNoClaim) return false;
+  take = __shfl_sync(kFullMask, take, 0);
+  uint64_t *q = gp.queues + (uint64_t)s * gp.bucket_cap;
+  const uint32_t idx = claim + lane;
+  uint64_t ent = ~0ull;
+  if ((uint32_t)lane < take) {
+    while ((ent = ld_relaxed_u64(q + idx)) == ~0ull) __nanosleep(20);  // producer mid-write
+    q[idx] = ~0ull;  // re-arm for the next launch
+  }
+  const int nv = (int)take;
+  (void)n;
+  const uint64_t a = ent != ~0ull ? reinterpret_cast<uint64_t>(gp.base[s]) + (ent >> 32) * (uint64_t)gp.row_bytes : 0ull;
+  if (sl.nslots) {  // through this warp's TMA slots, like the inline rows
+    __syncwarp();
+    if (lane < nv) {
+      s_addr[lane] = a;
+      s_idx[lane] = (uint32_t)ent;
+    }
+    __syncwarp();
+    sl.feed(s_addr, s_idx, (uint32_t)nv, 0, (uint32_t)nv, gp.out, gp.row_bytes, lane);
+    __syncwarp();
+  } else if (nv) {
+    copy_addr_rows<kStreamRegRows>(gp.out, gp.row_bytes, a, (uint32_t)ent, nv, lane);
+  }
+  return true;
+}
+
+template <typename KeyT>
+__device__ __forceinline__ void stream_body(const LocateParams &lp, const GatherParams &gp, uint32_t *s_dyn,
+                                            uint32_t pos) {
+  __shared__ uint32_t s_inl[kMaxSrc];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t n = lp.n, chunk = 32u * (uint32_t)gp.stream_k, nchunks = (n + chunk - 1) / chunk;
+  uint64_t *s_addr = reinterpret_cast<uint64_t *>(s_dyn) + warp * kStreamChunk;
+  uint32_t *s_idx = reinterpret_cast<uint32_t *>(s_dyn + 2 * kGatherWarps * kStreamChunk) + warp * kStreamChunk;
+  __shared__ __align__(8) uint64_t s_slot_bars[kGatherWarps][32];
+  if (threadIdx.x < kMaxSrc) s_inl[threadIdx.x] = 0;
+  StreamSlots sl;
+  sl.init(reinterpret_cast<uint8_t *>(s_dyn) + kRangeTabBytes + warp * kBulkWarpBytes, s_slot_bars[warp],
+          gp.row_bytes, lane, gp.stream_bulk != 0, gp.stream_host_cap, (uint32_t)gp.stream_nap);
+  __syncthreads();
+  // roles of the queued sources, as in gather_body: [host | peer_0 | ... | local]
+  const int host_src = gp.num_src - 1;
+  const int H = gp.inline_host ? 0 : gp.host_sms;
+  const int P = gp.inline_peer ? 0 : gp.peer_sms;
+  int my_src = -1;
+  if ((int)pos < H) {
+    if (warp < gp.host_warps) my_src = host_src;
+  } else if ((int)pos - H < gp.n_peers * P) {
+    my_src = gp.peer_src[((int)pos - H) / P];
+  }
+  Ctrl *ctrl = gp.ctrl;
+  // chunk claims: dynamic (atomic cursor, input order over time) or static (warp gw takes
+  // chunks gw, gw + W, ...: every warp works on the same window of keys at a time)
+  uint32_t static_next = pos * kGatherWarps + warp;
+  const uint32_t static_stride = gridDim.x * kGatherWarps;
+  auto claim_chunk = [&]() -> uint32_t {
+    uint32_t c = kNoClaim;
+    if (gp.stream_static) {
+      c = static_next;
+      static_next += static_stride;
+    } else if (lane == 0 && ld_relaxed_u32(&ctrl->chunk_cursor) < nchunks) {
+      c = atomicAdd(&ctrl->chunk_cursor, 1u);
+    }
+    return __shfl_sync(kFullMask, c, 0);
+  };
+  if (my_src < 0) {  // locating warp: chunks until none are left
+    while (true) {
+      const uint32_t c = claim_chunk();
+      if (c >= nchunks) break;
+      stream_chunk<KeyT>(lp, gp, c, lane, s_addr, s_idx, s_inl, sl);
+    }
+  } else {  // dedicated warp: drain my source's queue; locate chunks while it is empty
+    bool chunks_left = true;
+    while (true) {
+      if (stream_consume(gp, my_src, n, lane, s_addr, s_idx, sl)) continue;
+      uint32_t c = chunks_left ? claim_chunk() : kNoClaim;
+      if (c >= nchunks) chunks_left = false;
+      if (c < nchunks) {
+        stream_chunk<KeyT>(lp, gp, c, lane, s_addr, s_idx, s_inl, sl);
+        continue;
+      }
+      int fin = 0;
+      if (lane == 0)
+        fin = ld_acquire_u32(&ctrl->keys_done) >= n &&
+              ld_relaxed_u32(&ctrl->qhead[my_src]) >= ld_relaxed_u32(&ctrl->counts[my_src]);
+      if (__shfl_sync(kFullMask, fin, 0)) break;
+      __nanosleep(64);
+    }
+  }
+  sl.drain(gp.out, gp.row_bytes, lane);
+  __syncthreads();
+  if (threadIdx.x < gp.num_src && s_inl[threadIdx.x]) atomicAdd(&ctrl->counts[threadIdx.x], s_inl[threadIdx.x]);
+  finish_launch(ctrl, gp.num_src, n, 1);
 }
 
 // ---------------------------------------------------------------------------- K1+K2 fused
@@ -751,6 +1164,19 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
   }
   if (pos == 0 && threadIdx.x == 0) gp.ctrl->t_located = globaltimer_ns();
   gather_body(gp, s_dyn);
+}
+
+// ---------------------------------------------------------------------------- K3
+// Single-pass extraction (stream_body): its own kernel, so its register allocation does
+// not constrain the locate | barrier | gather kernel's.  Cooperative launch, one CTA per SM.
+template <typename KeyT>
+__global__ void __launch_bounds__(kGatherThreads, 1)
+    stream_extract_kernel(const LocateParams lp, const GatherParams gp) {
+  extern __shared__ __align__(16) uint32_t s_dyn[];
+  uint32_t smid;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+  const uint32_t pos = smid < (uint32_t)kMaxSmId ? gp.sm_pos[smid] : blockIdx.x;
+  stream_body<KeyT>(lp, gp, s_dyn, pos);
 }
 
 // ---------------------------------------------------------------------------- K2'
@@ -805,7 +1231,7 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
   __syncthreads();
   if (threadIdx.x < p.num_src && s_cnt[threadIdx.x])
     atomicAdd(&p.ctrl->counts[threadIdx.x], s_cnt[threadIdx.x]);
-  finish_launch(p.ctrl, p.num_src);
+  finish_launch(p.ctrl, p.num_src, p.n, 0);
 }
 
 // ---------------------------------------------------------------------------- probe

@@ -7,6 +7,7 @@
 #include <sys/mman.h>
 
 #include <algorithm>
+#include <cstddef>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -60,6 +61,7 @@ struct ugache_ctx {
   void *d_out_stage = nullptr;
   size_t out_stage_bytes = 0;
   uint64_t *d_host_sorted = nullptr;
+  uint64_t *d_queues = nullptr;  // single-pass queues, num_src x bucket_cap, ~0 between launches
   uint32_t *d_ranges = nullptr;  // 2 * kMaxRanges counters
   uint32_t range_shift = 0, n_ranges = 1;
   int host_sort = 1;
@@ -72,6 +74,9 @@ struct ugache_ctx {
   int fused = 2;                             // UGACHE_OPT_FUSED: 0 off, 1 on, 2 auto
   int early_walk = 0;                        // UGACHE_OPT_EARLY_WALK (env UGACHE_EARLY_WALK)
   int local_bulk = 2;                        // UGACHE_OPT_LOCAL_BULK (0 off, 1 on, 2 auto, 3)
+  int stream = 2;                            // UGACHE_OPT_STREAM (0 off, 1 on, 2 auto)
+  int inline_mask = UGACHE_INLINE_HOST;      // UGACHE_OPT_INLINE
+  int stream_k = 1, stream_host_last = 0, stream_host_cap = 0, stream_static = 1, stream_nap = 100;  // single-pass env knobs
   int host_warps = ugk::kHostWarps;  // env UGACHE_HOST_WARPS (A0 calibration knob)
   int stage_host_io = 0;             // env UGACHE_STAGE_HOST_IO=1: stage pinned host I/O too
   std::vector<int> smids;  // sorted %smid values of the device (one per SM)
@@ -82,6 +87,8 @@ struct ugache_ctx {
   bool timing = false;
   bool timing_valid = false;
   bool last_fused = false;  // last timed extract ran K1+K2 as one launch
+  bool last_single_pass = false;  // last timed extract ran the single pass (K3)
+  uint32_t *h_mirror = nullptr;  // pinned {n, host count, launches} of the last launch (Ctrl)
   cudaEvent_t ev[3] = {};
   int last_launches = 0;
   // message-based baseline: 0 idle, 1 local part done (buckets valid), 2 requests packed
@@ -100,6 +107,8 @@ namespace {
 constexpr size_t kOneCtaPerSmSmem = ugk::kGatherSmem;
 // UGACHE_OPT_FUSED = auto: batches up to this many keys run K1 + K2 in one launch.
 constexpr uint64_t kFusedAutoMaxKeys = 1u << 20;
+// UGACHE_OPT_STREAM = auto: the single pass only for rows up to this size.
+constexpr uint32_t kStreamAutoMaxRow = 1024;
 
 std::mutex g_reg_mu;
 std::map<const void *, int> g_reg_count;  // host-table registrations owned by this library
@@ -219,8 +228,14 @@ ugache_status ensure_scratch(ugache_ctx *ctx, uint64_t n) {
     cudaFree(ctx->d_host_sorted);
     ctx->d_host_sorted = nullptr;
   }
+  if (ctx->d_queues) {
+    cudaFree(ctx->d_queues);
+    ctx->d_queues = nullptr;
+  }
   const size_t bytes = (size_t)(ctx->cfg.num_gpus + 1) * cap * sizeof(uint64_t);
   UG_CUDA(ctx, cudaMalloc(&ctx->d_buckets, bytes));
+  UG_CUDA(ctx, cudaMalloc(&ctx->d_queues, bytes));
+  UG_CUDA(ctx, cudaMemset(ctx->d_queues, 0xFF, bytes));
   UG_CUDA(ctx, cudaMalloc(&ctx->d_host_sorted, cap * sizeof(uint64_t)));
   ctx->bucket_cap = cap;
   return UGACHE_OK;
@@ -356,6 +371,15 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   ctx->h_slot_keys.assign(slots.begin(), slots.begin() + (ptrdiff_t)ctx->n_slots);
   UG_CUDA(ctx, cudaMalloc(&ctx->d_ctrl, sizeof(ugk::Ctrl)));
   UG_CUDA(ctx, cudaMemset(ctx->d_ctrl, 0, sizeof(ugk::Ctrl)));
+  {  // pinned mirror of the last launch's {n, host count, launches} (path choice, K3)
+    UG_CUDA(ctx, cudaHostAlloc(reinterpret_cast<void **>(&ctx->h_mirror), 4 * sizeof(uint32_t),
+                               cudaHostAllocMapped));
+    std::memset(ctx->h_mirror, 0, 4 * sizeof(uint32_t));
+    void *dm = nullptr;
+    UG_CUDA(ctx, cudaHostGetDevicePointer(&dm, ctx->h_mirror, 0));
+    UG_CUDA(ctx, cudaMemcpy(reinterpret_cast<uint8_t *>(ctx->d_ctrl) + offsetof(ugk::Ctrl, host_mirror), &dm,
+                            sizeof(dm), cudaMemcpyHostToDevice));
+  }
   UG_CUDA(ctx, cudaMalloc(&ctx->d_ranges, 2 * ugk::kMaxRanges * sizeof(uint32_t)));
   UG_CUDA(ctx, cudaMemset(ctx->d_ranges, 0, 2 * ugk::kMaxRanges * sizeof(uint32_t)));
   // host key ranges: the smallest power-of-two rows per range giving <= kMaxRanges ranges
@@ -374,6 +398,12 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_EARLY_WALK")) ctx->early_walk = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_LOCAL_BULK")) ctx->local_bulk = std::max(0, std::min(3, atoi(e)));
   if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_STREAM_K")) ctx->stream_k = std::max(1, std::min(ugk::kStreamK, atoi(e)));
+  if (const char *e = getenv("UGACHE_STREAM_HOST_LAST")) ctx->stream_host_last = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_STREAM_NAP")) ctx->stream_nap = std::max(0, atoi(e));
+  if (const char *e = getenv("UGACHE_STREAM_STATIC")) ctx->stream_static = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_STREAM_HOST_CAP")) ctx->stream_host_cap = std::max(0, atoi(e));
+  if (const char *e = getenv("UGACHE_STREAM")) ctx->stream = std::max(0, std::min(2, atoi(e)));
   if (const char *e = getenv("UGACHE_HOST_WARPS")) ctx->host_warps = std::max(1, std::min(ugk::kGatherWarps, atoi(e)));
   for (int i = 0; i < 3; ++i) UG_CUDA(ctx, cudaEventCreate(&ctx->ev[i]));
   ctx->src_base[cfg->rank] = ctx->slab;
@@ -405,6 +435,10 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   UG_CUDA(ctx, cudaFuncSetAttribute(ugk::fused_extract_kernel<int64_t>,
                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem));
   UG_CUDA(ctx, cudaFuncSetAttribute(ugk::fused_extract_kernel<uint32_t>,
+                                    cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem));
+  UG_CUDA(ctx, cudaFuncSetAttribute(ugk::stream_extract_kernel<int64_t>,
+                                    cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem));
+  UG_CUDA(ctx, cudaFuncSetAttribute(ugk::stream_extract_kernel<uint32_t>,
                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem));
   UG_CUDA(ctx, cudaFuncSetAttribute(ugk::random_dispatch_kernel<int64_t>,
                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem));
@@ -772,6 +806,14 @@ ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value) 
       if (value < 0 || value > 3) return UGACHE_EINVAL;
       ctx->local_bulk = (int)value;
       return UGACHE_OK;
+    case UGACHE_OPT_STREAM:
+      if (value < 0 || value > 2) return UGACHE_EINVAL;
+      ctx->stream = (int)value;
+      return UGACHE_OK;
+    case UGACHE_OPT_INLINE:
+      if (value < 0 || value > (UGACHE_INLINE_HOST | UGACHE_INLINE_PEERS)) return UGACHE_EINVAL;
+      ctx->inline_mask = (int)value;
+      return UGACHE_OK;
     case UGACHE_OPT_DEDICATION:
       if (value != UGACHE_DEDICATE_SMS && value != UGACHE_DEDICATE_WARPS) return UGACHE_EINVAL;
       ctx->warp_dedication = value == UGACHE_DEDICATE_WARPS;
@@ -893,6 +935,15 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     gp.host_warps = ctx->host_warps;
     gp.local_bulk = R <= ugk::kBulkWarpBytes / 2 ? ctx->local_bulk : 0;
     gp.early_walk = ctx->early_walk && ctx->host_walk && ctx->host_sort && !ctx->warp_dedication && !msg_local;
+    gp.inline_host = (ctx->inline_mask & UGACHE_INLINE_HOST) != 0;
+    gp.inline_peer = (ctx->inline_mask & UGACHE_INLINE_PEERS) != 0;
+    gp.queues = ctx->d_queues;
+    gp.stream_bulk = R <= ugk::kBulkWarpBytes / 2 && ctx->local_bulk != 0;
+    gp.stream_k = ctx->stream_k;
+    gp.stream_host_last = ctx->stream_host_last;
+    gp.stream_host_cap = ctx->stream_host_cap;
+    gp.stream_static = ctx->stream_static;
+    gp.stream_nap = ctx->stream_nap;
     int grid = 0;
     build_roles(ctx, &gp, &grid);
     if (msg_local) {  // message baseline: no SM reads a peer; the peer buckets stay for msg_*
@@ -900,8 +951,31 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
       gp.peer_sms = 0;
       gp.host_sms_max = ctx->host_dynamic ? std::max(ctx->host_sms, gp.num_sms) : ctx->host_sms;
     }
+    // single pass unless the last launch on this ctx (its counts mirrored to pinned host
+    // memory by the kernel) had a host bucket dense enough for range-ordered reads; rows
+    // above 1 KB stay on the two-phase path (measured faster there)
+    bool stream = !msg_local && !ctx->warp_dedication && ctx->stream != 0;
+    if (stream && ctx->stream == 2) {
+      const volatile uint32_t *m = ctx->h_mirror;
+      const uint64_t pn = m[0], ph = m[1];
+      stream = R <= kStreamAutoMaxRow &&
+               !(m[2] && pn && ctx->host_sort && ph * n >= (uint64_t)ctx->host_sort_min * pn);
+    }
     const bool fused = ctx->fused == 1 || (ctx->fused == 2 && n <= kFusedAutoMaxKeys);
-    if (fused) {  // K1 + K2 in one cooperative launch
+    if (stream) {  // K3: one cooperative launch, no grid barrier
+      if (ctx->timing) {
+        UG_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
+        UG_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
+      }
+      void *kargs[] = {&lp, &gp};
+      const void *fn = key_type == UGACHE_KEY_I64 ? (const void *)ugk::stream_extract_kernel<int64_t>
+                                                  : (const void *)ugk::stream_extract_kernel<uint32_t>;
+      UG_CUDA(ctx, cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(ugk::kGatherThreads), kargs,
+                                               kOneCtaPerSmSmem, s));
+      ctx->last_launches = 1;
+      ctx->last_fused = false;
+      ctx->last_single_pass = true;
+    } else if (fused) {  // K1 + K2 in one cooperative launch
       if (ctx->timing) {
         UG_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
         UG_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
@@ -913,6 +987,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
                                                kOneCtaPerSmSmem, s));
       ctx->last_launches = 1;
       ctx->last_fused = true;
+      ctx->last_single_pass = false;
     } else {
       const unsigned lgrid = (unsigned)((n + ugk::kLocateTile - 1) / ugk::kLocateTile);
       if (ctx->timing) UG_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
@@ -927,6 +1002,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
                                                dim3(ugk::kGatherThreads), kargs, kOneCtaPerSmSmem, s));
       ctx->last_launches = 2;
       ctx->last_fused = false;
+      ctx->last_single_pass = false;
     }
   }
   if (ctx->timing) {
@@ -1084,7 +1160,10 @@ ugache_status ugache_last_batch_timing(ugache_ctx *ctx, float *ms_locate, float 
   float a = 0, b = 0;
   UG_CUDA(ctx, cudaEventElapsedTime(&a, ctx->ev[0], ctx->ev[1]));
   UG_CUDA(ctx, cudaEventElapsedTime(&b, ctx->ev[1], ctx->ev[2]));
-  if (ctx->last_fused && ctx->mode == UGACHE_MODE_FACTORED) {
+  if (ctx->last_single_pass && ctx->mode == UGACHE_MODE_FACTORED) {
+    b += a;  // single pass: no separate locate phase
+    a = 0.f;
+  } else if (ctx->last_fused && ctx->mode == UGACHE_MODE_FACTORED) {
     // one launch: split it at the grid barrier with the kernel's own %globaltimer stamps
     ugk::Ctrl c;
     UG_CUDA(ctx, cudaMemcpy(&c, ctx->d_ctrl, sizeof(c), cudaMemcpyDeviceToHost));
@@ -1143,6 +1222,8 @@ ugache_status ugache_destroy(ugache_ctx *ctx) {
     cudaFree(ctx->d_keys_stage);
     cudaFree(ctx->d_out_stage);
     cudaFree(ctx->d_host_sorted);
+    cudaFree(ctx->d_queues);
+    if (ctx->h_mirror) cudaFreeHost(ctx->h_mirror);
     cudaFree(ctx->d_ranges);
     cudaFree(ctx->d_loc_new);
     cudaFree(ctx->d_refresh);

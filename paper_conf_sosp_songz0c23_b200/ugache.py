@@ -205,6 +205,16 @@ class UGache:
         """'off' (two launches), 'on' (one cooperative launch) or 'auto'."""
         self.set_option(_abi.OPT_FUSED, {"off": 0, "on": 1, "auto": 2}[mode])
 
+    def set_stream(self, mode):
+        """Single-pass extraction: 'off', 'on' or 'auto' (default: unless the previous
+        batch's host bucket was dense)."""
+        self.set_option(_abi.OPT_STREAM, {"off": 0, "on": 1, "auto": 2}[mode])
+
+    def set_inline(self, host: bool = True, peers: bool = False):
+        """Single pass: which non-local sources the locating warps copy themselves."""
+        self.set_option(_abi.OPT_INLINE, (_abi.INLINE_HOST if host else 0) |
+                        (_abi.INLINE_PEERS if peers else 0))
+
     def set_host_walk(self, on: bool):
         self.set_option(_abi.OPT_HOST_WALK, int(on))
 

@@ -215,10 +215,12 @@ def test_timing_and_repeated_extracts(torch_cuda):
     t, (c,) = make_group(torch_cuda, wl.num_rows, 512, wl.capacity_rows, 1, h)
     c.enable_timing(True)
     keys = synth.make_batch(wl, 0, 5)
-    for _ in range(20):  # counters re-armed by the kernel itself across launches
+    for i in range(20):  # counters re-armed by the kernel itself across launches
+        c.set_stream("on" if i % 2 else "off")
         per = check_batch(torch_cuda, c, t, keys, wl.num_rows, 512, 1)
         a, b = c.last_batch_timing()
-        assert a > 0 and b > 0
+        # the single pass has no separate locate phase: it is reported as 0
+        assert b > 0 and (a == 0 if i % 2 else a > 0)
     c.close()
 
 
@@ -486,21 +488,22 @@ def test_sparse_host_walk_parity(torch_cuda, G, walk, key_dtype):
         c.close()
 
 
-@pytest.mark.parametrize("fused", ["on", "off"])
+@pytest.mark.parametrize("fused", ["on", "off", "stream"])
 @pytest.mark.parametrize("G,C,n", [(1, 3000, 1), (1, 3000, 40_000), (4, 2000, 50_001), (3, 40_000, 9_999)])
 def test_fused_and_split_launch_parity(torch_cuda, fused, G, C, n):
-    """K1+K2 in one cooperative launch (grid barrier) vs two launches: same bytes/counts,
-    dense and sparse host buckets, ragged sizes, u32 keys."""
+    """K1+K2 in one cooperative launch (grid barrier) vs two launches vs the single pass:
+    same bytes/counts, dense and sparse host buckets, ragged sizes, u32 keys."""
     N, R = 300_000, 512
     h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(41).permutation(N)]
     t, group = make_group(torch_cuda, N, R, C, G, h)
     keys = np.random.default_rng(42).integers(-2, N + 2, n)
     for g, c in enumerate(group):
-        c.set_fused(fused)
+        c.set_fused("on" if fused == "stream" else fused)
+        c.set_stream("on" if fused == "stream" else "off")
         c.set_local_bulk(g % 2 == 0)
         for kd in (np.int64, np.uint32):
             check_batch(torch_cuda, c, t, np.abs(keys) if kd == np.uint32 else keys, N, R, G, key_dtype=kd)
-            assert c.last_launch_count() == (1 if fused == "on" else 2)
+            assert c.last_launch_count() == (2 if fused == "off" else 1)
     for c in group:
         c.close()
 
@@ -556,11 +559,94 @@ def test_early_host_walk_parity(torch_cuda, early, G, C, n):
     rng = np.random.default_rng(44)
     for g, c in enumerate(group):
         c.set_fused("on")
+        c.set_stream("off")
         c.set_early_walk(early)
         for b in range(3):  # repeated launches: the walk cursor is re-armed by the kernel
             keys = rng.integers(0, N, n)
             keys[:: 997] = N + 1
             per = check_batch(torch_cuda, c, t, keys, N, R, G)
             assert per[G] > 0
+    for c in group:
+        c.close()
+
+
+@pytest.mark.parametrize("inline", ["host", "none", "all"])
+@pytest.mark.parametrize("G,host_sms,peer_sms", [(1, 12, 0), (1, 148, 0), (2, 12, 60), (4, 1, 1),
+                                                 (8, 12, 19), (8, 1, 21)])
+def test_single_pass_parity(torch_cuda, inline, G, host_sms, peer_sms):
+    """Single-pass extraction (UGACHE_OPT_STREAM): locate + inline local copies + per-source
+    queues drained by dedicated SMs.  Every dedication split, including grids whose every SM
+    is dedicated (1 + 7 x 21 = 148: every warp is a consumer that also locates), inline and
+    queued host / peer rows, ragged and empty chunks, out-of-range keys, u32 keys, and
+    repeated launches (queues re-armed to ~0 by their consumers)."""
+    N, R = 200_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(45).permutation(N)]
+    t, group = make_group(torch_cuda, N, R, 6000, G, h)
+    rng = np.random.default_rng(46)
+    for g, c in enumerate(group[:3]):
+        c.set_fused("on")
+        c.set_stream("on")
+        c.set_inline(host=inline != "none", peers=inline == "all")
+        if G > 1 or host_sms != 12:
+            c.set_dedication(host_sms, peer_sms if G > 1 else 0)
+        for b, n in enumerate([1, 63, 64, 65, 5_000, 100_001, 77_777]):
+            c.set_local_bulk(b != 6)  # rows through TMA slots, or the register path
+            keys = rng.integers(0, N, n)
+            keys[:: 613] = N + b
+            kd = np.uint32 if b % 2 else np.int64
+            per = check_batch(torch_cuda, c, t, keys, N, R, G, key_dtype=kd)
+            assert c.last_launch_count() == 1
+            if n > 50_000:
+                assert per[G] > 0 and (G == 1 or per[[j for j in range(G) if j != g]].sum() > 0)
+    for c in group:
+        c.close()
+
+
+def test_stream_auto_switches_on_host_density(torch_cuda):
+    """UGACHE_OPT_STREAM = auto picks the path from the previous launch's host count (mirrored
+    by the kernel to pinned host memory): a dense-host batch after sparse ones (and back)
+    stays bit-exact, and the path taken follows the density (single pass: no locate phase)."""
+    N, R = 300_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(47).permutation(N)]
+    t, (c,) = make_group(torch_cuda, N, R, 30_000, 1, h)
+    c.set_fused("on")
+    c.set_stream("auto")
+    c.enable_timing(True)
+    rng = np.random.default_rng(48)
+    loc, _ = c.export_placement()
+    host_keys = np.nonzero((loc >> 56) == 1)[0]
+    local_keys = np.nonzero((loc >> 56) == 0)[0]
+    prev_dense = False
+    for b in range(7):
+        dense = b in (2, 3, 4)
+        keys = rng.choice(host_keys if dense else local_keys, 200_000)
+        if not dense:
+            keys[:50] = host_keys[:50]
+        per = check_batch(torch_cuda, c, t, keys, N, R, 1)
+        assert per[1] == (200_000 if dense else 50)
+        a, _ = c.last_batch_timing()
+        assert (a > 0) == prev_dense   # ordered path after a dense batch, single pass otherwise
+        prev_dense = dense
+    c.close()
+
+
+@pytest.mark.parametrize("G", [1, 4])
+@pytest.mark.parametrize("k", ["1", "2"])
+def test_single_pass_static_schedule_and_chunk_sizes(torch_cuda, monkeypatch, G, k):
+    """Single pass with the static chunk schedule (UGACHE_STREAM_STATIC) and both chunk
+    sizes (UGACHE_STREAM_K), queued peers and inline host rows."""
+    monkeypatch.setenv("UGACHE_STREAM_STATIC", "1")
+    monkeypatch.setenv("UGACHE_STREAM_K", k)
+    N, R = 200_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(49).permutation(N)]
+    t, group = make_group(torch_cuda, N, R, 6000, G, h)
+    rng = np.random.default_rng(50)
+    for g, c in enumerate(group[:2]):
+        c.set_fused("on")
+        c.set_stream("on")
+        for n in (1, 100, 60_001, 300_000):
+            keys = rng.integers(0, N, n)
+            keys[::101] = N + 9
+            check_batch(torch_cuda, c, t, keys, N, R, G)
     for c in group:
         c.close()

@@ -1,8 +1,11 @@
+# Round-end style check on one B200: build, GPU tests, smoke, default bench, reference arm.
 set -x
-mkdir -p gpurun_out/r1e
-nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/r1e/smi.txt
-python __graft_entry__.py > gpurun_out/r1e/build.txt 2>&1
-timeout 900 python -m pytest tests -m gpu -x -q > gpurun_out/r1e/pytest_gpu.txt 2>&1; echo "pytest rc $?" >> gpurun_out/r1e/pytest_gpu.txt
-timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/r1e/smoke.txt 2>&1; echo "smoke rc $?" >> gpurun_out/r1e/smoke.txt
-timeout 900 python bench.py > gpurun_out/r1e/bench.json 2> gpurun_out/r1e/bench.err
-tail -3 gpurun_out/r1e/bench.json
+o=${1:-gpurun_out/check}; mkdir -p $o
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > $o/smi.txt
+nproc > $o/nproc.txt; free -g >> $o/nproc.txt
+python __graft_entry__.py > $o/build.txt 2>&1
+timeout 900 python -m pytest tests -m gpu -x -q > $o/pytest_gpu.txt 2>&1; echo "pytest rc $?" >> $o/pytest_gpu.txt
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $o/smoke.txt 2>&1; echo "smoke rc $?" >> $o/smoke.txt
+timeout 900 python bench.py > $o/bench.json 2> $o/bench.err
+timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > $o/bench_ref.json 2> $o/bench_ref.err
+tail -2 $o/pytest_gpu.txt; tail -c 600 $o/bench.json
