@@ -141,6 +141,7 @@ struct GatherParams {
   int32_t stream_host_cap;         // single pass: non-local rows in flight per warp (0 = slots)
   int32_t stream_static;           // single pass: static chunk schedule instead of the cursor
   int32_t stream_nap;              // single pass: ns a warp sleeps when all its slots are in flight
+  int32_t stream_prefetch;         // single pass: locating warps prefetch the next chunks' keys/entries
 };
 
 struct RandomParams {
@@ -1099,7 +1100,29 @@ __device__ __forceinline__ void stream_body(const LocateParams &lp, const Gather
     }
     return __shfl_sync(kFullMask, c, 0);
   };
-  if (my_src < 0) {  // locating warp: chunks until none are left
+  if (my_src < 0 && gp.stream_prefetch) {
+    // locating warp, software-pipelined two deep: the keys of chunk i+2 and the location
+    // entries of chunk i+1 are in flight while chunk i's rows are fed to the slots
+    KeyT k1[kStreamK];
+    uint64_t e0[kStreamK], e1[kStreamK];
+    uint32_t c0 = claim_chunk(), c1 = kNoClaim;
+    if (c0 < nchunks) {
+      stream_keys<KeyT>(lp, gp, c0, lane, k1);
+      stream_locs<KeyT>(lp, gp, c0, lane, k1, e0);
+      c1 = claim_chunk();
+      if (c1 < nchunks) stream_keys<KeyT>(lp, gp, c1, lane, k1);
+    }
+    while (c0 < nchunks) {
+      if (c1 < nchunks) stream_locs<KeyT>(lp, gp, c1, lane, k1, e1);
+      const uint32_t c2 = c1 < nchunks ? claim_chunk() : kNoClaim;
+      if (c2 < nchunks) stream_keys<KeyT>(lp, gp, c2, lane, k1);
+      stream_chunk_located<KeyT>(lp, gp, c0, e0, lane, s_addr, s_idx, s_inl, sl);
+      c0 = c1;
+      c1 = c2;
+#pragma unroll
+      for (int it = 0; it < kStreamK; ++it) e0[it] = e1[it];
+    }
+  } else if (my_src < 0) {  // locating warp: chunks until none are left
     while (true) {
       const uint32_t c = claim_chunk();
       if (c >= nchunks) break;

@@ -76,7 +76,8 @@ struct ugache_ctx {
   int local_bulk = 2;                        // UGACHE_OPT_LOCAL_BULK (0 off, 1 on, 2 auto, 3)
   int stream = 2;                            // UGACHE_OPT_STREAM (0 off, 1 on, 2 auto)
   int inline_mask = UGACHE_INLINE_HOST;      // UGACHE_OPT_INLINE
-  int stream_k = 1, stream_host_last = 0, stream_host_cap = 0, stream_static = 1, stream_nap = 100;  // single-pass env knobs
+  int stream_k = 1, stream_host_last = 0, stream_host_cap = 0, stream_static = 1, stream_nap = 100,
+      stream_prefetch = 0;  // single-pass env knobs
   int host_warps = ugk::kHostWarps;  // env UGACHE_HOST_WARPS (A0 calibration knob)
   int stage_host_io = 0;             // env UGACHE_STAGE_HOST_IO=1: stage pinned host I/O too
   std::vector<int> smids;  // sorted %smid values of the device (one per SM)
@@ -400,6 +401,7 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_STREAM_K")) ctx->stream_k = std::max(1, std::min(ugk::kStreamK, atoi(e)));
   if (const char *e = getenv("UGACHE_STREAM_HOST_LAST")) ctx->stream_host_last = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_STREAM_PREFETCH")) ctx->stream_prefetch = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_STREAM_NAP")) ctx->stream_nap = std::max(0, atoi(e));
   if (const char *e = getenv("UGACHE_STREAM_STATIC")) ctx->stream_static = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_STREAM_HOST_CAP")) ctx->stream_host_cap = std::max(0, atoi(e));
@@ -944,6 +946,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     gp.stream_host_cap = ctx->stream_host_cap;
     gp.stream_static = ctx->stream_static;
     gp.stream_nap = ctx->stream_nap;
+    gp.stream_prefetch = ctx->stream_prefetch;
     int grid = 0;
     build_roles(ctx, &gp, &grid);
     if (msg_local) {  // message baseline: no SM reads a peer; the peer buckets stay for msg_*
