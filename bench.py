@@ -325,7 +325,7 @@ def main():
     torch.cuda.synchronize()
     clocks = Clocks(local) if (rank == 0 and not args.no_clocks) else None  # every GPU of the node
     time.sleep(0.3 if clocks else 0)
-    evs, loc_ms, gat_ms, per_src = [], [], [], []
+    evs, loc_ms, gat_ms, per_src, paths = [], [], [], [], []
     launches = 0
     for i in range(args.steps):
         evs.append(step(args.warmup + i, True))
@@ -335,6 +335,7 @@ def main():
         per, _ = cache.last_batch_stats()
         per_src.append(per)
         launches += cache.last_launch_count()
+        paths.append(cache.last_extract_path())
     stream.synchronize()
     torch.cuda.synchronize()
     ugdist.barrier()
@@ -440,13 +441,20 @@ def main():
     kern_ms = [a + b for a, b in zip(loc_ms, gat_ms)] if launches == args.steps else list(gat_ms)
     gat_s = statistics.mean(kern_ms) / 1e3
     loc_s = statistics.mean(loc_ms) / 1e3
-    # algorithmic bytes of the timed kernel: rows read per source + rows written + bucket
-    # reads; with K1+K2 fused (one launch per step) also K1's key + location entry + bucket
-    # write per key (2R + 8 + 8 + 16 per key)
-    fused = launches == args.steps
-    kname = "fused_extract_kernel" if fused else "factored_gather_kernel"
+    # algorithmic bytes of the timed kernel: rows read per source + rows
+    # written + key + location entry per key, plus the bucket traffic of the path taken:
+    #   fused K1+K2 (one launch): 16 B/key (bucket write + read);
+    #   split: K2 alone is timed (8 B/key bucket read; K1 is its own launch);
+    #   single pass K3: no local bucket -- only queued (peer) rows take 16 B
+    path = statistics.mode(paths)
+    kname = {"single_pass": "stream_extract_kernel", "fused": "fused_extract_kernel"}.get(
+        path, "factored_gather_kernel")
+    fused = path in ("fused", "single_pass")
     k1_hbm_bytes = n * (kb + 8 + 8)
-    gather_hbm_bytes = n_local * R + n * R + n * 8 + (k1_hbm_bytes if fused else 0)
+    if path == "single_pass":
+        gather_hbm_bytes = n_local * R + n * R + n * (kb + 8) + n_peer * 16
+    else:
+        gather_hbm_bytes = n_local * R + n * R + n * 8 + (k1_hbm_bytes if fused else 0)
     gather_pcie_bytes = n_host * R
     t_hbm = gather_hbm_bytes / (hbm * 1e9)
     t_pcie = gather_pcie_bytes / (pcie * 1e9) if pcie else 0.0
@@ -463,14 +471,16 @@ def main():
         achieved, peak, unit, psrc = n_peer * R / gat_s / 1e9, nvl, "GB/s", \
             "B200_PROFILING.md measured peer copy"
     # whole-step source-mix roofline (locate + gather): every byte the step moves
-    step_hbm = n_local * R + n * R + n * 8 + k1_hbm_bytes
+    step_hbm = gather_hbm_bytes if path == "single_pass" else n_local * R + n * R + n * 8 + k1_hbm_bytes
     t_roof = max(step_hbm / (hbm * 1e9), t_pcie, t_nvl)
     ms_per_step = statistics.mean(step_ms)
     traffic = traffic_pcie = traffic_src = None
     try:  # per-launch DRAM traffic of K2 from the committed ncu capture of this workload
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
             rec = json.load(f)[wl.name][kname]
-        traffic, traffic_pcie, traffic_src = rec["dram_bytes"], rec.get("pcie_read_bytes"), rec["source"]
+        c_run = args.cache_ratio if args.cache_ratio is not None else wl.cache_ratio
+        if abs(rec.get("cache_ratio", wl.cache_ratio) - c_run) < 1e-9:  # same workload only
+            traffic, traffic_pcie, traffic_src = rec["dram_bytes"], rec.get("pcie_read_bytes"), rec["source"]
     except Exception:
         pass
     line = {
@@ -483,7 +493,9 @@ def main():
                      "traffic_pcie_read": traffic_pcie, "traffic_source": traffic_src,
                      "algorithmic_bytes": {"hbm": gather_hbm_bytes, "pcie": gather_pcie_bytes,
                                            "nvlink": n_peer * R},
-                     "kernel": kname + (" (K1 locate+bucket and K2 gather, one cooperative launch)" if fused else ""),
+                     "kernel": kname + {"fused": " (K1 locate+bucket and K2 gather, one cooperative launch)",
+                                        "single_pass": " (K3: locate + copy in one pass, no grid barrier)"}.get(path, ""),
+                     "path": path,
                      "peak_source": psrc,
                      "kernel_ms": statistics.mean(kern_ms)},
         "source_mix_roofline": {"t_roof_us": t_roof * 1e6, "t_step_us": ms_per_step * 1e3,

@@ -343,6 +343,13 @@ ugache_status ugache_last_batch_timing(ugache_ctx *ctx, float *ms_locate, float 
 /* Number of kernel launches the last extract issued (for launch accounting). */
 ugache_status ugache_last_launch_count(const ugache_ctx *ctx, int32_t *launches);
 
+/* Which path the last extract took (roofline accounting): UGACHE_PATH_NONE (n = 0),
+ * UGACHE_PATH_SPLIT (K1 + K2, two launches), UGACHE_PATH_FUSED (K1 + grid barrier + K2, one
+ * cooperative launch), UGACHE_PATH_SINGLE_PASS (K3), UGACHE_PATH_RANDOM (unfactored K2'). */
+enum { UGACHE_PATH_NONE = 0, UGACHE_PATH_SPLIT = 1, UGACHE_PATH_FUSED = 2, UGACHE_PATH_SINGLE_PASS = 3,
+       UGACHE_PATH_RANDOM = 4 };
+ugache_status ugache_last_extract_path(const ugache_ctx *ctx, int32_t *path);
+
 /* Copy out this GPU's location table (N entries) and slot list (capacity entries) for the
  * placement checker.  Synchronous. */
 ugache_status ugache_export_placement(ugache_ctx *ctx, uint64_t *loc, uint64_t *slot_keys,

@@ -28,6 +28,7 @@ OPT_HOST_ORDERING, OPT_STAGE_HOST_IO, OPT_HOST_WARPS = 0, 1, 2
 OPT_DEDICATION, OPT_WARP_HOST, OPT_WARP_PEER, OPT_HOST_WALK, OPT_FUSED = 3, 4, 5, 6, 7
 OPT_LOCAL_BULK, OPT_EARLY_WALK, OPT_STREAM, OPT_INLINE = 8, 9, 10, 11
 INLINE_HOST, INLINE_PEERS = 1, 2
+PATHS = {0: "none", 1: "split", 2: "fused", 3: "single_pass", 4: "random"}
 DEDICATE_SMS, DEDICATE_WARPS = 0, 1
 FLAG_HOST_TIER = 1
 
@@ -96,6 +97,7 @@ SIGNATURES = {
     "ugache_enable_timing": (_ST, [_P, _c.c_int32]),
     "ugache_last_batch_timing": (_ST, [_P, ctypes.POINTER(_c.c_float), ctypes.POINTER(_c.c_float)]),
     "ugache_last_launch_count": (_ST, [_P, ctypes.POINTER(_c.c_int32)]),
+    "ugache_last_extract_path": (_ST, [_P, ctypes.POINTER(_c.c_int32)]),
     "ugache_export_placement": (_ST, [_P, _P, _P, ctypes.POINTER(_c.c_uint64)]),
     "ugache_read_slab": (_ST, [_P, _c.c_uint64, _c.c_uint64, _P]),
     "ugache_destroy": (_ST, [_P]),

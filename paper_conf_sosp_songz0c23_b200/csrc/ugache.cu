@@ -1185,6 +1185,16 @@ ugache_status ugache_last_launch_count(const ugache_ctx *ctx, int32_t *launches)
   return UGACHE_OK;
 }
 
+ugache_status ugache_last_extract_path(const ugache_ctx *ctx, int32_t *path) {
+  if (!ctx || !path) return UGACHE_EINVAL;
+  if (ctx->last_launches == 0) *path = UGACHE_PATH_NONE;
+  else if (ctx->mode == UGACHE_MODE_RANDOM_DISPATCH) *path = UGACHE_PATH_RANDOM;
+  else if (ctx->last_single_pass) *path = UGACHE_PATH_SINGLE_PASS;
+  else if (ctx->last_fused) *path = UGACHE_PATH_FUSED;
+  else *path = UGACHE_PATH_SPLIT;
+  return UGACHE_OK;
+}
+
 ugache_status ugache_export_placement(ugache_ctx *ctx, uint64_t *loc, uint64_t *slot_keys,
                                       uint64_t *n_slots) {
   if (!ctx) return UGACHE_EINVAL;

@@ -275,6 +275,13 @@ class UGache:
               self.ctx)
         return n.value
 
+    def last_extract_path(self) -> str:
+        """'split', 'fused', 'single_pass', 'random' or 'none' (ugache_last_extract_path)."""
+        p = ctypes.c_int32()
+        check(lib().ugache_last_extract_path(self.ctx, ctypes.byref(p)), "ugache_last_extract_path",
+              self.ctx)
+        return _abi.PATHS[p.value]
+
     def export_placement(self):
         loc = np.empty(self.num_rows, dtype=np.uint64)
         slots = np.empty(max(self.plan.capacity_rows, 1), dtype=np.uint64)

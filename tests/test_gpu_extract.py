@@ -504,6 +504,7 @@ def test_fused_and_split_launch_parity(torch_cuda, fused, G, C, n):
         for kd in (np.int64, np.uint32):
             check_batch(torch_cuda, c, t, np.abs(keys) if kd == np.uint32 else keys, N, R, G, key_dtype=kd)
             assert c.last_launch_count() == (2 if fused == "off" else 1)
+            assert c.last_extract_path() == {"off": "split", "on": "fused", "stream": "single_pass"}[fused]
     for c in group:
         c.close()
 
@@ -626,6 +627,7 @@ def test_stream_auto_switches_on_host_density(torch_cuda):
         assert per[1] == (200_000 if dense else 50)
         a, _ = c.last_batch_timing()
         assert (a > 0) == prev_dense   # ordered path after a dense batch, single pass otherwise
+        assert c.last_extract_path() == ("fused" if prev_dense else "single_pass")
         prev_dense = dense
     c.close()
 
