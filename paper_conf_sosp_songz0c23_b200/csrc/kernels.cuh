@@ -142,6 +142,7 @@ struct GatherParams {
   int32_t stream_static;           // single pass: static chunk schedule instead of the cursor
   int32_t stream_nap;              // single pass: ns a warp sleeps when all its slots are in flight
   int32_t stream_prefetch;         // single pass: locating warps prefetch the next chunks' keys/entries
+  int32_t stream_queues;           // single pass: some source is queued (consumers exist)
 };
 
 struct RandomParams {
@@ -929,6 +930,7 @@ __device__ __forceinline__ void stream_chunk_located(const LocateParams &lp, con
   const int host_src = gp.num_src - 1;
   int s[kStreamK];
   uint32_t nbad = 0;
+  bool any_queued = false;
 #pragma unroll
   for (int it = 0; it < kStreamK; ++it) {
     const uint32_t i = i0 + it * 32 + lane;
@@ -944,6 +946,7 @@ __device__ __forceinline__ void stream_chunk_located(const LocateParams &lp, con
     const int si = s[it];
     const bool inl = si >= 0 && (si == gp.local_src || (si == host_src ? gp.inline_host : gp.inline_peer));
     const int qs = (si >= 0 && !inl) ? si : -1;
+    any_queued |= __any_sync(kFullMask, qs >= 0);
     // queued rows: warp-aggregated reservation on the source's queue, then the entry
     const uint32_t qpeers = __match_any_sync(kFullMask, qs);
     const int qleader = __ffs(qpeers) - 1;
@@ -993,10 +996,16 @@ __device__ __forceinline__ void stream_chunk_located(const LocateParams &lp, con
     }
   }
   __syncwarp();
-  // this chunk's reservations and queue entries precede its keys_done increment
-  __threadfence();
-  __syncwarp();
-  if (lane == 0) atomicAdd(&gp.ctrl->keys_done, min(chunk, n - i0));
+  // keys_done only serves consumers (a queue is final once every key is located); with no
+  // queued source in this launch nobody reads it.  A chunk that reserved queue entries
+  // orders the reservations before its increment; one that reserved none needs no fence.
+  if (gp.stream_queues) {
+    if (any_queued) {
+      __threadfence();
+      __syncwarp();
+    }
+    if (lane == 0) atomicAdd(&gp.ctrl->keys_done, min(chunk, n - i0));
+  }
 }
 
 template <typename KeyT>
@@ -1088,15 +1097,26 @@ __device__ __forceinline__ void stream_body(const LocateParams &lp, const Gather
   Ctrl *ctrl = gp.ctrl;
   // chunk claims: dynamic (atomic cursor, input order over time) or static (warp gw takes
   // chunks gw, gw + W, ...: every warp works on the same window of keys at a time)
+  // stream_static >= 2: static for the full rounds of W chunks but the last (stream_static
+  // - 2), then the dynamic cursor for the remaining chunks (balances the tail)
   uint32_t static_next = pos * kGatherWarps + warp;
   const uint32_t static_stride = gridDim.x * kGatherWarps;
+  uint32_t static_end = 0;
+  if (gp.stream_static == 1) {
+    static_end = nchunks;
+  } else if (gp.stream_static >= 2) {
+    const uint32_t rounds = nchunks / static_stride, keep = (uint32_t)(gp.stream_static - 2);
+    static_end = (rounds > keep ? rounds - keep : 0) * static_stride;
+  }
   auto claim_chunk = [&]() -> uint32_t {
     uint32_t c = kNoClaim;
-    if (gp.stream_static) {
+    if (static_next < static_end) {
       c = static_next;
       static_next += static_stride;
-    } else if (lane == 0 && ld_relaxed_u32(&ctrl->chunk_cursor) < nchunks) {
-      c = atomicAdd(&ctrl->chunk_cursor, 1u);
+    } else if (gp.stream_static == 1) {
+      c = kNoClaim;
+    } else if (lane == 0 && static_end + ld_relaxed_u32(&ctrl->chunk_cursor) < nchunks) {
+      c = static_end + atomicAdd(&ctrl->chunk_cursor, 1u);
     }
     return __shfl_sync(kFullMask, c, 0);
   };

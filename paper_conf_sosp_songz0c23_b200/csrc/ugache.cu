@@ -403,7 +403,7 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_STREAM_HOST_LAST")) ctx->stream_host_last = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_STREAM_PREFETCH")) ctx->stream_prefetch = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_STREAM_NAP")) ctx->stream_nap = std::max(0, atoi(e));
-  if (const char *e = getenv("UGACHE_STREAM_STATIC")) ctx->stream_static = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_STREAM_STATIC")) ctx->stream_static = std::max(0, atoi(e));
   if (const char *e = getenv("UGACHE_STREAM_HOST_CAP")) ctx->stream_host_cap = std::max(0, atoi(e));
   if (const char *e = getenv("UGACHE_STREAM")) ctx->stream = std::max(0, std::min(2, atoi(e)));
   if (const char *e = getenv("UGACHE_HOST_WARPS")) ctx->host_warps = std::max(1, std::min(ugk::kGatherWarps, atoi(e)));
@@ -947,6 +947,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     gp.stream_static = ctx->stream_static;
     gp.stream_nap = ctx->stream_nap;
     gp.stream_prefetch = ctx->stream_prefetch;
+    gp.stream_queues = (!gp.inline_host && ctx->host_sms > 0) || (!gp.inline_peer && ctx->cfg.num_gpus > 1);
     int grid = 0;
     build_roles(ctx, &gp, &grid);
     if (msg_local) {  // message baseline: no SM reads a peer; the peer buckets stay for msg_*

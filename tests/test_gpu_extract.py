@@ -634,10 +634,12 @@ def test_stream_auto_switches_on_host_density(torch_cuda):
 
 @pytest.mark.parametrize("G", [1, 4])
 @pytest.mark.parametrize("k", ["1", "2"])
-def test_single_pass_static_schedule_and_chunk_sizes(torch_cuda, monkeypatch, G, k):
-    """Single pass with the static chunk schedule (UGACHE_STREAM_STATIC) and both chunk
-    sizes (UGACHE_STREAM_K), queued peers and inline host rows."""
-    monkeypatch.setenv("UGACHE_STREAM_STATIC", "1")
+@pytest.mark.parametrize("sched", ["0", "1", "2", "3"])
+def test_single_pass_static_schedule_and_chunk_sizes(torch_cuda, monkeypatch, G, k, sched):
+    """Single pass with every chunk schedule (UGACHE_STREAM_STATIC: 0 dynamic cursor, 1
+    static, 2/3 static rounds then a dynamic tail), both chunk sizes (UGACHE_STREAM_K),
+    queued peers and inline host rows."""
+    monkeypatch.setenv("UGACHE_STREAM_STATIC", sched)
     monkeypatch.setenv("UGACHE_STREAM_K", k)
     N, R = 200_000, 512
     h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(49).permutation(N)]
