@@ -1216,9 +1216,15 @@ template <typename KeyT>
 __global__ void __launch_bounds__(kGatherThreads, 1)
     stream_extract_kernel(const LocateParams lp, const GatherParams gp) {
   extern __shared__ __align__(16) uint32_t s_dyn[];
-  uint32_t smid;
-  asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-  const uint32_t pos = smid < (uint32_t)kMaxSmId ? gp.sm_pos[smid] : blockIdx.x;
+  // With queued sources the CTA's role is its SM's (cooperative launch, one CTA per SM);
+  // without, no warp ever waits on another, the launch is a plain one and CTA b takes
+  // position b of the static chunk schedule.
+  uint32_t pos = blockIdx.x;
+  if (gp.stream_queues) {
+    uint32_t smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    pos = smid < (uint32_t)kMaxSmId ? gp.sm_pos[smid] : blockIdx.x;
+  }
   stream_body<KeyT>(lp, gp, s_dyn, pos);
 }
 

@@ -77,7 +77,7 @@ struct ugache_ctx {
   int stream = 2;                            // UGACHE_OPT_STREAM (0 off, 1 on, 2 auto)
   int inline_mask = UGACHE_INLINE_HOST;      // UGACHE_OPT_INLINE
   int stream_k = 1, stream_host_last = 0, stream_host_cap = 0, stream_static = 1, stream_nap = 100,
-      stream_prefetch = 0;  // single-pass env knobs
+      stream_prefetch = 0, stream_coop = 0;  // single-pass env knobs
   int host_warps = ugk::kHostWarps;  // env UGACHE_HOST_WARPS (A0 calibration knob)
   int stage_host_io = 0;             // env UGACHE_STAGE_HOST_IO=1: stage pinned host I/O too
   std::vector<int> smids;  // sorted %smid values of the device (one per SM)
@@ -401,6 +401,7 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_STREAM_K")) ctx->stream_k = std::max(1, std::min(ugk::kStreamK, atoi(e)));
   if (const char *e = getenv("UGACHE_STREAM_HOST_LAST")) ctx->stream_host_last = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_STREAM_COOP")) ctx->stream_coop = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_STREAM_PREFETCH")) ctx->stream_prefetch = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_STREAM_NAP")) ctx->stream_nap = std::max(0, atoi(e));
   if (const char *e = getenv("UGACHE_STREAM_STATIC")) ctx->stream_static = std::max(0, atoi(e));
@@ -974,8 +975,12 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
       void *kargs[] = {&lp, &gp};
       const void *fn = key_type == UGACHE_KEY_I64 ? (const void *)ugk::stream_extract_kernel<int64_t>
                                                   : (const void *)ugk::stream_extract_kernel<uint32_t>;
-      UG_CUDA(ctx, cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(ugk::kGatherThreads), kargs,
-                                               kOneCtaPerSmSmem, s));
+      if (gp.stream_queues || ctx->stream_coop) {
+        UG_CUDA(ctx, cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(ugk::kGatherThreads), kargs,
+                                                 kOneCtaPerSmSmem, s));
+      } else {  // no queues: no CTA waits on another, a plain launch is enough
+        UG_CUDA(ctx, cudaLaunchKernel(fn, dim3(grid), dim3(ugk::kGatherThreads), kargs, kOneCtaPerSmSmem, s));
+      }
       ctx->last_launches = 1;
       ctx->last_fused = false;
       ctx->last_single_pass = true;
