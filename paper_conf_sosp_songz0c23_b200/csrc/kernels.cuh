@@ -137,6 +137,8 @@ struct GatherParams {
   uint64_t *queues;                // num_src x bucket_cap entries, ~0 between launches
   int32_t stream_bulk;             // single pass: inline rows through TMA slots (StreamSlots)
   int32_t stream_k;                // single pass: keys per lane per chunk (1 or 2)
+  int32_t stream_ck;               // single pass: lanes holding a key per step (32; 4..16 for
+                                   // small batches, so every warp gets a chunk)
   int32_t stream_host_last;        // single pass: non-local inline rows after the local ones
   int32_t stream_host_cap;         // single pass: non-local rows in flight per warp (0 = slots)
   int32_t stream_static;           // single pass: static chunk schedule instead of the cursor
@@ -901,22 +903,23 @@ template <typename KeyT>
 __device__ __forceinline__ void stream_keys(const LocateParams &lp, const GatherParams &gp, uint32_t c, int lane,
                                             KeyT (&k)[kStreamK]) {
   const KeyT *keys = static_cast<const KeyT *>(lp.keys);
-  const uint32_t K = (uint32_t)gp.stream_k, i0 = c * 32u * K;
+  const uint32_t K = (uint32_t)gp.stream_k, ck = (uint32_t)gp.stream_ck, i0 = c * ck * K;
 #pragma unroll
   for (int it = 0; it < kStreamK; ++it) {
-    const uint32_t i = i0 + it * 32 + lane;
-    k[it] = (it < (int)K && i < lp.n) ? keys[i] : (KeyT)0;
+    const uint32_t i = i0 + it * ck + lane;
+    k[it] = (it < (int)K && (uint32_t)lane < ck && i < lp.n) ? keys[i] : (KeyT)0;
   }
 }
 template <typename KeyT>
 __device__ __forceinline__ void stream_locs(const LocateParams &lp, const GatherParams &gp, uint32_t c, int lane,
                                             const KeyT (&k)[kStreamK], uint64_t (&e)[kStreamK]) {
-  const uint32_t K = (uint32_t)gp.stream_k, i0 = c * 32u * K;
+  const uint32_t K = (uint32_t)gp.stream_k, ck = (uint32_t)gp.stream_ck, i0 = c * ck * K;
 #pragma unroll
   for (int it = 0; it < kStreamK; ++it) {
-    const uint32_t i = i0 + it * 32 + lane;
-    e[it] = (it < (int)K && i < lp.n && key_in_range<KeyT>(k[it], lp.num_rows)) ? ld_nc_u64(lp.loc + (uint64_t)k[it])
-                                                                               : ~0ull;
+    const uint32_t i = i0 + it * ck + lane;
+    e[it] = (it < (int)K && (uint32_t)lane < ck && i < lp.n && key_in_range<KeyT>(k[it], lp.num_rows))
+                ? ld_nc_u64(lp.loc + (uint64_t)k[it])
+                : ~0ull;
   }
 }
 
@@ -925,7 +928,7 @@ template <typename KeyT>
 __device__ __forceinline__ void stream_chunk_located(const LocateParams &lp, const GatherParams &gp, uint32_t c,
                                                      const uint64_t (&e)[kStreamK], int lane, uint64_t *s_addr,
                                                      uint32_t *s_idx, uint32_t *s_inl, StreamSlots &sl) {
-  const uint32_t K = (uint32_t)gp.stream_k, chunk = 32u * K;
+  const uint32_t K = (uint32_t)gp.stream_k, ck = (uint32_t)gp.stream_ck, chunk = ck * K;
   const uint32_t R = gp.row_bytes, n = lp.n, i0 = c * chunk;
   const int host_src = gp.num_src - 1;
   int s[kStreamK];
@@ -933,9 +936,9 @@ __device__ __forceinline__ void stream_chunk_located(const LocateParams &lp, con
   bool any_queued = false;
 #pragma unroll
   for (int it = 0; it < kStreamK; ++it) {
-    const uint32_t i = i0 + it * 32 + lane;
+    const uint32_t i = i0 + it * ck + lane;
     s[it] = -1;
-    if (it < (int)K && i < n) {
+    if (it < (int)K && (uint32_t)lane < ck && i < n) {
       if (e[it] != ~0ull) {
         s[it] = (int)(e[it] >> UGACHE_LOC_SRC_SHIFT);
       } else {
@@ -978,7 +981,7 @@ __device__ __forceinline__ void stream_chunk_located(const LocateParams &lp, con
       if (take) {
         const uint32_t at = nl + __popc(m & lanemask_lt());
         s_addr[at] = reinterpret_cast<uint64_t>(gp.base[si]) + (e[it] & UGACHE_LOC_ROW_MASK) * (uint64_t)R;
-        s_idx[at] = i0 + it * 32 + lane;
+        s_idx[at] = i0 + it * ck + lane;
       }
       nl += __popc(m);
     }
@@ -1075,7 +1078,8 @@ __device__ __forceinline__ void stream_body(const LocateParams &lp, const Gather
                                             uint32_t pos) {
   __shared__ uint32_t s_inl[kMaxSrc];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const uint32_t n = lp.n, chunk = 32u * (uint32_t)gp.stream_k, nchunks = (n + chunk - 1) / chunk;
+  const uint32_t n = lp.n, chunk = (uint32_t)gp.stream_ck * (uint32_t)gp.stream_k,
+                 nchunks = (n + chunk - 1) / chunk;
   uint64_t *s_addr = reinterpret_cast<uint64_t *>(s_dyn) + warp * kStreamChunk;
   uint32_t *s_idx = reinterpret_cast<uint32_t *>(s_dyn + 2 * kGatherWarps * kStreamChunk) + warp * kStreamChunk;
   __shared__ __align__(8) uint64_t s_slot_bars[kGatherWarps][32];

@@ -943,6 +943,17 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     gp.queues = ctx->d_queues;
     gp.stream_bulk = R <= ugk::kBulkWarpBytes / 2 && ctx->local_bulk != 0;
     gp.stream_k = ctx->stream_k;
+    gp.stream_ck = 32;
+    {  // small batches: fewer keys per chunk, so that every warp of the grid gets one
+      const uint64_t warps = (uint64_t)ctx->sm_count * ugk::kGatherWarps;
+      const uint64_t per = (n + warps - 1) / warps;
+      if (per < 32) {
+        uint32_t ck = 4;
+        while (ck < per) ck <<= 1;
+        gp.stream_ck = (int32_t)ck;
+        gp.stream_k = 1;
+      }
+    }
     gp.stream_host_last = ctx->stream_host_last;
     gp.stream_host_cap = ctx->stream_host_cap;
     gp.stream_static = ctx->stream_static;
