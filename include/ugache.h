@@ -300,7 +300,8 @@ typedef enum {
  *   Rows move through per-lane TMA shared-memory slots (cp.async.bulk in and out, up to
  *   12 KB in flight per warp).  No grid barrier and no bucket round trip for local rows.
  *   0 = off (locate | grid barrier | factored gather); 1 = always; 2 (default) = for rows of
- *   at most 1 KB, unless the last launch on this ctx had a host bucket dense enough for
+ *   at most 1 KB and no queued peer source (G = 1, or UGACHE_INLINE_PEERS), unless the last
+ *   launch on this ctx had a host bucket dense enough for
  *   range-ordered reads (scaled to this batch's size; the kernel mirrors its counts to
  *   pinned host memory, so the choice needs no synchronisation).  Ignored with
  *   UGACHE_DEDICATE_WARPS and on the message path.  Timing reports the whole launch as

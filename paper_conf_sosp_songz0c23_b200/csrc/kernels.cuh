@@ -145,6 +145,8 @@ struct GatherParams {
   int32_t stream_nap;              // single pass: ns a warp sleeps when all its slots are in flight
   int32_t stream_prefetch;         // single pass: locating warps prefetch the next chunks' keys/entries
   int32_t stream_queues;           // single pass: some source is queued (consumers exist)
+  uint64_t queue_cap;              // single pass: entries per source in `queues`
+  uint32_t *qctr;                  // single pass: [2][kMaxSrc][kMaxSmId] sub-queue counts / heads
 };
 
 struct RandomParams {
@@ -899,6 +901,26 @@ struct StreamSlots {
   }
 };
 
+// Sub-queues (single pass): the queue of source s is split into one sub-queue per CTA
+// dedicated to s, so each is drained by one CTA's warps (no grid-wide claim contention):
+// chunk c's rows of s go to sub-queue c mod P_s, of capacity ceil(nchunks / P_s) * chunk.
+__device__ __forceinline__ int stream_role_ctas(const GatherParams &gp, int s) {
+  if (s == gp.num_src - 1) return gp.inline_host ? 0 : gp.host_sms;
+  return gp.inline_peer ? 0 : gp.peer_sms;
+}
+__device__ __forceinline__ uint32_t *sub_count(const GatherParams &gp, int s, int j) {
+  return gp.qctr + (uint32_t)s * kMaxSmId + (uint32_t)j;
+}
+__device__ __forceinline__ uint32_t *sub_head(const GatherParams &gp, int s, int j) {
+  return gp.qctr + (uint32_t)(kMaxSrc + s) * kMaxSmId + (uint32_t)j;
+}
+__device__ __forceinline__ uint64_t *sub_queue(const GatherParams &gp, int s, int j, uint32_t nchunks,
+                                               uint32_t chunk) {
+  const uint32_t P = (uint32_t)stream_role_ctas(gp, s);
+  const uint64_t cap = (uint64_t)((nchunks + P - 1) / P) * chunk;
+  return gp.queues + (uint64_t)s * gp.queue_cap + (uint64_t)j * cap;
+}
+
 template <typename KeyT>
 __device__ __forceinline__ void stream_keys(const LocateParams &lp, const GatherParams &gp, uint32_t c, int lane,
                                             KeyT (&k)[kStreamK]) {
@@ -954,10 +976,11 @@ __device__ __forceinline__ void stream_chunk_located(const LocateParams &lp, con
     const uint32_t qpeers = __match_any_sync(kFullMask, qs);
     const int qleader = __ffs(qpeers) - 1;
     uint32_t b = 0;
-    if (qs >= 0 && lane == qleader) b = atomicAdd(&gp.ctrl->counts[qs], (uint32_t)__popc(qpeers));
+    const int qj = qs >= 0 ? (int)(c % (uint32_t)stream_role_ctas(gp, qs)) : 0;
+    if (qs >= 0 && lane == qleader) b = atomicAdd(sub_count(gp, qs, qj), (uint32_t)__popc(qpeers));
     b = __shfl_sync(kFullMask, b, qleader);
     if (qs >= 0)
-      st_relaxed_u64(gp.queues + (uint64_t)qs * gp.bucket_cap + b + __popc(qpeers & lanemask_lt()),
+      st_relaxed_u64(sub_queue(gp, qs, qj, (n + chunk - 1) / chunk, chunk) + b + __popc(qpeers & lanemask_lt()),
                      ((e[it] & UGACHE_LOC_ROW_MASK) << 32) | (uint64_t)i);
     // inline rows: per-CTA statistics
     const int is = inl ? si : -1;
@@ -1021,23 +1044,25 @@ __device__ __forceinline__ void stream_chunk(const LocateParams &lp, const Gathe
   stream_chunk_located<KeyT>(lp, gp, c, e, lane, s_addr, s_idx, s_inl, sl);
 }
 
-// Dedicated warp: claim up to kRowsInFlight (register path: kStreamRegRows) entries of
-// source s's queue and copy them.
+// Dedicated warp: claim up to one entry per TMA slot (register path: kStreamRegRows) of
+// source s's sub-queue j and copy them.
 // Returns false when nothing was reserved beyond the queue head.
-__device__ __forceinline__ bool stream_consume(const GatherParams &gp, int s, uint32_t n, int lane,
-                                               uint64_t *s_addr, uint32_t *s_idx, StreamSlots &sl) {
-  Ctrl *ctrl = gp.ctrl;
+__device__ __forceinline__ bool stream_consume(const GatherParams &gp, int s, int j, uint32_t nchunks,
+                                               uint32_t chunk, int lane, uint64_t *s_addr, uint32_t *s_idx,
+                                               StreamSlots &sl) {
   // Claims never pass the reservation counter (CAS), so every claimed entry is being
   // written by a producer that does not block: waiting for it cannot deadlock even when
   // every warp of the grid is a consumer.
   uint32_t claim = kNoClaim, take = 0;
   if (lane == 0) {
-    uint32_t h = ld_relaxed_u32(&ctrl->qhead[s]);
+    uint32_t *head = sub_head(gp, s, j);
+    const uint32_t *count = sub_count(gp, s, j);
+    uint32_t h = ld_relaxed_u32(head);
     while (true) {
-      const uint32_t c = ld_relaxed_u32(&ctrl->counts[s]);
+      const uint32_t c = ld_relaxed_u32(count);
       if (h >= c) break;
-      const uint32_t t = min(sl.nslots ? (uint32_t)kRowsInFlight : (uint32_t)kStreamRegRows, c - h);
-      const uint32_t old = atomicCAS(&ctrl->qhead[s], h, h + t);
+      const uint32_t t = min(sl.nslots ? (uint32_t)sl.nslots : (uint32_t)kStreamRegRows, c - h);
+      const uint32_t old = atomicCAS(head, h, h + t);
       if (old == h) {
         claim = h, take = t;
         break;
@@ -1048,7 +1073,7 @@ __device__ __forceinline__ bool stream_consume(const GatherParams &gp, int s, ui
   claim = __shfl_sync(kFullMask, claim, 0);
   if (claim == kNoClaim) return false;
   take = __shfl_sync(kFullMask, take, 0);
-  uint64_t *q = gp.queues + (uint64_t)s * gp.bucket_cap;
+  uint64_t *q = sub_queue(gp, s, j, nchunks, chunk);
   const uint32_t idx = claim + lane;
   uint64_t ent = ~0ull;
   if ((uint32_t)lane < take) {
@@ -1056,7 +1081,6 @@ __device__ __forceinline__ bool stream_consume(const GatherParams &gp, int s, ui
     q[idx] = ~0ull;  // re-arm for the next launch
   }
   const int nv = (int)take;
-  (void)n;
   const uint64_t a = ent != ~0ull ? reinterpret_cast<uint64_t>(gp.base[s]) + (ent >> 32) * (uint64_t)gp.row_bytes : 0ull;
   if (sl.nslots) {  // through this warp's TMA slots, like the inline rows
     __syncwarp();
@@ -1092,12 +1116,13 @@ __device__ __forceinline__ void stream_body(const LocateParams &lp, const Gather
   const int host_src = gp.num_src - 1;
   const int H = gp.inline_host ? 0 : gp.host_sms;
   const int P = gp.inline_peer ? 0 : gp.peer_sms;
-  int my_src = -1;
+  int role_src = -1, role_j = 0;  // this CTA's queued source and its sub-queue
   if ((int)pos < H) {
-    if (warp < gp.host_warps) my_src = host_src;
+    role_src = host_src, role_j = (int)pos;
   } else if ((int)pos - H < gp.n_peers * P) {
-    my_src = gp.peer_src[((int)pos - H) / P];
+    role_src = gp.peer_src[((int)pos - H) / P], role_j = ((int)pos - H) % P;
   }
+  const int my_src = (role_src == host_src && warp >= gp.host_warps) ? -1 : role_src;
   Ctrl *ctrl = gp.ctrl;
   // chunk claims: dynamic (atomic cursor, input order over time) or static (warp gw takes
   // chunks gw, gw + W, ...: every warp works on the same window of keys at a time)
@@ -1155,7 +1180,7 @@ __device__ __forceinline__ void stream_body(const LocateParams &lp, const Gather
   } else {  // dedicated warp: drain my source's queue; locate chunks while it is empty
     bool chunks_left = true;
     while (true) {
-      if (stream_consume(gp, my_src, n, lane, s_addr, s_idx, sl)) continue;
+      if (stream_consume(gp, my_src, role_j, nchunks, chunk, lane, s_addr, s_idx, sl)) continue;
       uint32_t c = chunks_left ? claim_chunk() : kNoClaim;
       if (c >= nchunks) chunks_left = false;
       if (c < nchunks) {
@@ -1165,7 +1190,7 @@ __device__ __forceinline__ void stream_body(const LocateParams &lp, const Gather
       int fin = 0;
       if (lane == 0)
         fin = ld_acquire_u32(&ctrl->keys_done) >= n &&
-              ld_relaxed_u32(&ctrl->qhead[my_src]) >= ld_relaxed_u32(&ctrl->counts[my_src]);
+              ld_relaxed_u32(sub_head(gp, my_src, role_j)) >= ld_relaxed_u32(sub_count(gp, my_src, role_j));
       if (__shfl_sync(kFullMask, fin, 0)) break;
       __nanosleep(64);
     }
@@ -1173,6 +1198,12 @@ __device__ __forceinline__ void stream_body(const LocateParams &lp, const Gather
   sl.drain(gp.out, gp.row_bytes, lane);
   __syncthreads();
   if (threadIdx.x < gp.num_src && s_inl[threadIdx.x]) atomicAdd(&ctrl->counts[threadIdx.x], s_inl[threadIdx.x]);
+  if (role_src >= 0 && threadIdx.x == 0) {  // my sub-queue is drained: publish its count, re-arm it
+    uint32_t *cnt = sub_count(gp, role_src, role_j);
+    atomicAdd(&ctrl->counts[role_src], *cnt);
+    *cnt = 0;
+    *sub_head(gp, role_src, role_j) = 0;
+  }
   finish_launch(ctrl, gp.num_src, n, 1);
 }
 

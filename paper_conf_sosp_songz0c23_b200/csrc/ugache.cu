@@ -61,7 +61,9 @@ struct ugache_ctx {
   void *d_out_stage = nullptr;
   size_t out_stage_bytes = 0;
   uint64_t *d_host_sorted = nullptr;
-  uint64_t *d_queues = nullptr;  // single-pass queues, num_src x bucket_cap, ~0 between launches
+  uint64_t *d_queues = nullptr;  // single-pass queues, num_src x queue_cap, ~0 between launches
+  uint64_t queue_cap = 0;
+  uint32_t *d_qctr = nullptr;    // single-pass sub-queue counts / heads, zero between launches
   uint32_t *d_ranges = nullptr;  // 2 * kMaxRanges counters
   uint32_t range_shift = 0, n_ranges = 1;
   int host_sort = 1;
@@ -235,8 +237,16 @@ ugache_status ensure_scratch(ugache_ctx *ctx, uint64_t n) {
   }
   const size_t bytes = (size_t)(ctx->cfg.num_gpus + 1) * cap * sizeof(uint64_t);
   UG_CUDA(ctx, cudaMalloc(&ctx->d_buckets, bytes));
-  UG_CUDA(ctx, cudaMalloc(&ctx->d_queues, bytes));
-  UG_CUDA(ctx, cudaMemset(ctx->d_queues, 0xFF, bytes));
+  // sub-queues round each one up to whole chunks: room for one extra chunk per sub-queue
+  ctx->queue_cap = cap + (uint64_t)(ctx->sm_count + 1) * ugk::kStreamChunk;
+  const size_t qbytes = (size_t)(ctx->cfg.num_gpus + 1) * ctx->queue_cap * sizeof(uint64_t);
+  UG_CUDA(ctx, cudaMalloc(&ctx->d_queues, qbytes));
+  UG_CUDA(ctx, cudaMemset(ctx->d_queues, 0xFF, qbytes));
+  if (!ctx->d_qctr) {
+    const size_t cb = 2 * (size_t)ugk::kMaxSrc * ugk::kMaxSmId * sizeof(uint32_t);
+    UG_CUDA(ctx, cudaMalloc(&ctx->d_qctr, cb));
+    UG_CUDA(ctx, cudaMemset(ctx->d_qctr, 0, cb));
+  }
   UG_CUDA(ctx, cudaMalloc(&ctx->d_host_sorted, cap * sizeof(uint64_t)));
   ctx->bucket_cap = cap;
   return UGACHE_OK;
@@ -941,6 +951,8 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     gp.inline_host = (ctx->inline_mask & UGACHE_INLINE_HOST) != 0;
     gp.inline_peer = (ctx->inline_mask & UGACHE_INLINE_PEERS) != 0;
     gp.queues = ctx->d_queues;
+    gp.queue_cap = ctx->queue_cap;
+    gp.qctr = ctx->d_qctr;
     gp.stream_bulk = R <= ugk::kBulkWarpBytes / 2 && ctx->local_bulk != 0;
     gp.stream_k = ctx->stream_k;
     gp.stream_ck = 32;
@@ -974,7 +986,10 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     if (stream && ctx->stream == 2) {
       const volatile uint32_t *m = ctx->h_mirror;
       const uint64_t pn = m[0], ph = m[1];
-      stream = R <= kStreamAutoMaxRow &&
+      // with peer rows queued to dedicated SMs the two-phase kernel measured faster (fake
+      // peers), so auto takes the single pass only without peer queues
+      const bool peer_queues = ctx->cfg.num_gpus > 1 && !(ctx->inline_mask & UGACHE_INLINE_PEERS);
+      stream = R <= kStreamAutoMaxRow && !peer_queues &&
                !(m[2] && pn && ctx->host_sort && ph * n >= (uint64_t)ctx->host_sort_min * pn);
     }
     const bool fused = ctx->fused == 1 || (ctx->fused == 2 && n <= kFusedAutoMaxKeys);
@@ -1253,6 +1268,7 @@ ugache_status ugache_destroy(ugache_ctx *ctx) {
     cudaFree(ctx->d_out_stage);
     cudaFree(ctx->d_host_sorted);
     cudaFree(ctx->d_queues);
+    cudaFree(ctx->d_qctr);
     if (ctx->h_mirror) cudaFreeHost(ctx->h_mirror);
     cudaFree(ctx->d_ranges);
     cudaFree(ctx->d_loc_new);

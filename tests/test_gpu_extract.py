@@ -654,3 +654,22 @@ def test_single_pass_static_schedule_and_chunk_sizes(torch_cuda, monkeypatch, G,
             check_batch(torch_cuda, c, t, keys, N, R, G)
     for c in group:
         c.close()
+
+
+def test_stream_auto_with_peers(torch_cuda):
+    """auto keeps the two-phase kernel when peer rows are queued to dedicated SMs (G > 1,
+    default) and takes the single pass once peers are inline; both bit-exact."""
+    N, R = 200_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(51).permutation(N)]
+    t, group = make_group(torch_cuda, N, R, 20_000, 2, h)
+    c = group[0]
+    c.set_stream("auto")
+    keys = np.random.default_rng(52).integers(0, N, 30_000)
+    for peers_inline, want in ((False, "fused"), (True, "single_pass")):
+        c.set_inline(host=True, peers=peers_inline)
+        for _ in range(2):
+            per = check_batch(torch_cuda, c, t, keys, N, R, 2)
+            assert per[1] > 0
+        assert c.last_extract_path() == want
+    for g in group:
+        g.close()
