@@ -5,6 +5,9 @@
 //  K2 factored_gather_kernel : one CTA per SM, CTA role = source; non-local roles copy
 //                            their bucket first, then every CTA pads the local bucket
 //                            through an atomic cursor (FEM)
+//  K3 stream_extract_kernel : single pass -- chunks located and copied at once through
+//                            per-lane TMA slots; queued sources drained by their dedicated
+//                            SMs from per-CTA sub-queues (no grid barrier, no local bucket)
 //  K2' random_dispatch_kernel : unfactored peer-based baseline, ablation only
 //  K5 fill_kernel          : Filler, host rows -> this GPU's cache slab
 //
@@ -146,6 +149,7 @@ struct GatherParams {
   int32_t stream_prefetch;         // single pass: locating warps prefetch the next chunks' keys/entries
   int32_t stream_queues;           // single pass: some source is queued (consumers exist)
   uint64_t queue_cap;              // single pass: entries per source in `queues`
+  int32_t stream_regstore;         // single pass: slots leave by warp-wide stores, not bulk copies
   uint32_t *qctr;                  // single pass: [2][kMaxSrc][kMaxSmId] sub-queue counts / heads
 };
 
@@ -832,10 +836,14 @@ struct StreamSlots {
   int nslots;         // 0: register path (copy_addr_rows)
   int slow_cap;       // max non-local rows in flight per warp
   uint32_t nap;       // ns to sleep when every slot is in flight
+  int regstore;       // landed rows leave by warp-wide 16-B stores instead of a bulk copy
+  uint8_t *wbase;     // slot 0 of this warp
 
   __device__ __forceinline__ void init(uint8_t *wbuf, uint64_t *wbars, uint32_t R, int lane, bool on, int cap,
-                                       uint32_t nap_ns) {
+                                       uint32_t nap_ns, int reg_store) {
     nap = nap_ns;
+    regstore = reg_store;
+    wbase = wbuf;
     nslots = on ? min(32, (int)(kBulkWarpBytes / R)) : 0;
     slow_cap = cap > 0 ? cap : 32;
     buf = wbuf + (uint32_t)lane * R;
@@ -861,14 +869,37 @@ struct StreamSlots {
     slow = 0;
     bulk_s2g(out + (uint64_t)oidx * R, buf, R, policy);
   }
+  // regstore: the whole warp copies every landed slot to out (16 B per lane per step) and
+  // the slots are free at once (no bulk store to wait for).
+  __device__ __forceinline__ void retire_warp(bool ready, uint8_t *out, uint32_t R, int lane) {
+    uint32_t m = __ballot_sync(kFullMask, ready);
+    if (!m) return;
+    const uint32_t V = R >> 4;
+    while (m) {
+      const int u = __ffs(m) - 1;
+      m &= m - 1;
+      const uint32_t o = __shfl_sync(kFullMask, oidx, u);
+      const uint8_t *src = wbase + (uint32_t)u * R;
+      for (uint32_t j = lane; j < V; j += 32)
+        st_cs_v4(out + (uint64_t)o * R + (uint64_t)j * 16u, *reinterpret_cast<const uint4 *>(src + j * 16u));
+    }
+    if (ready) {
+      phase ^= 1u;
+      busy = 0;
+      slow = 0;
+    }
+    __syncwarp();
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // reads before the next TMA writes
+  }
   // Copy list entries [0, nl): free lanes take the next entries in list order; entries
   // [sb, se) are non-local rows, at most slow_cap of them in flight per warp.
   __device__ __forceinline__ void feed(const uint64_t *s_addr, const uint32_t *s_idx, uint32_t nl,
                                        uint32_t sb, uint32_t se, uint8_t *out, uint32_t R, int lane) {
     uint32_t next = 0;
     while (next < nl) {
-      const bool free_lane = lane < nslots && !busy;  // free before this round's retirements
-      if (lane < nslots && busy && landed()) retire(out, R);
+      if (regstore) retire_warp(lane < nslots && busy && landed(), out, R, lane);
+      const bool free_lane = lane < nslots && !busy;  // free before this round's bulk retirements
+      if (!regstore && lane < nslots && busy && landed()) retire(out, R);
       const uint32_t fm = __ballot_sync(kFullMask, free_lane);
       const uint32_t in_slow = (uint32_t)__popc(__ballot_sync(kFullMask, busy && slow));
       uint32_t t = min((uint32_t)__popc(fm), nl - next);
@@ -881,7 +912,7 @@ struct StreamSlots {
       }
       const uint32_t e = next + __popc(fm & lanemask_lt());
       if (free_lane && e < next + t) {
-        bulk_wait_read_all();  // this lane's previous store has left the slot
+        if (!regstore) bulk_wait_read_all();  // this lane's previous store has left the slot
         oidx = s_idx[e];
         slow = e >= sb && e < se;
         mbar_expect_tx(bar, R);
@@ -892,7 +923,10 @@ struct StreamSlots {
     }
   }
   __device__ __forceinline__ void drain(uint8_t *out, uint32_t R, int lane) {
-    if (lane < nslots && busy) {
+    if (regstore) {
+      if (lane < nslots && busy) mbar_wait(bar, phase);
+      retire_warp(lane < nslots && busy, out, R, lane);
+    } else if (lane < nslots && busy) {
       mbar_wait(bar, phase);
       retire(out, R);
     }
@@ -1110,7 +1144,8 @@ __device__ __forceinline__ void stream_body(const LocateParams &lp, const Gather
   if (threadIdx.x < kMaxSrc) s_inl[threadIdx.x] = 0;
   StreamSlots sl;
   sl.init(reinterpret_cast<uint8_t *>(s_dyn) + kRangeTabBytes + warp * kBulkWarpBytes, s_slot_bars[warp],
-          gp.row_bytes, lane, gp.stream_bulk != 0, gp.stream_host_cap, (uint32_t)gp.stream_nap);
+          gp.row_bytes, lane, gp.stream_bulk != 0, gp.stream_host_cap, (uint32_t)gp.stream_nap,
+          gp.stream_regstore);
   __syncthreads();
   // roles of the queued sources, as in gather_body: [host | peer_0 | ... | local]
   const int host_src = gp.num_src - 1;

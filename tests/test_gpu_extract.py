@@ -674,3 +674,22 @@ def test_stream_auto_with_peers(torch_cuda):
         assert c.last_extract_path() == want
     for g in group:
         g.close()
+
+
+@pytest.mark.parametrize("G", [1, 4])
+def test_single_pass_register_store_retire(torch_cuda, monkeypatch, G):
+    """Single pass with landed slots leaving by warp-wide 16-B stores (UGACHE_STREAM_REGSTORE)
+    instead of bulk copies: bit-exact incl. 1536-B rows (8 slots per warp)."""
+    monkeypatch.setenv("UGACHE_STREAM_REGSTORE", "1")
+    for R in (512, 1536):
+        N = 100_000
+        h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(53).permutation(N)]
+        t, group = make_group(torch_cuda, N, R, 8000, G, h)
+        c = group[0]
+        c.set_stream("on")
+        c.set_inline(host=True, peers=G > 2)
+        for n in (5, 20_000, 120_001):
+            keys = np.random.default_rng(n).integers(0, N + 3, n)
+            check_batch(torch_cuda, c, t, keys, N, R, G)
+        for g in group:
+            g.close()
