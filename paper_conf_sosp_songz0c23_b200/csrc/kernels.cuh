@@ -150,6 +150,7 @@ struct GatherParams {
   int32_t stream_queues;           // single pass: some source is queued (consumers exist)
   uint64_t queue_cap;              // single pass: entries per source in `queues`
   int32_t stream_regstore;         // single pass: slots leave by warp-wide stores, not bulk copies
+  int32_t stream_peer_warps;       // single pass: consumer warps per peer-dedicated CTA
   uint32_t *qctr;                  // single pass: [2][kMaxSrc][kMaxSmId] sub-queue counts / heads
 };
 
@@ -1157,7 +1158,10 @@ __device__ __forceinline__ void stream_body(const LocateParams &lp, const Gather
   } else if ((int)pos - H < gp.n_peers * P) {
     role_src = gp.peer_src[((int)pos - H) / P], role_j = ((int)pos - H) % P;
   }
-  const int my_src = (role_src == host_src && warp >= gp.host_warps) ? -1 : role_src;
+  // consumer warps of a dedicated CTA: host_warps (host) / stream_peer_warps (peers); the
+  // CTA's other warps locate chunks like everyone else
+  const int consumers = role_src == host_src ? gp.host_warps : gp.stream_peer_warps;
+  const int my_src = warp < consumers ? role_src : -1;
   Ctrl *ctrl = gp.ctrl;
   // chunk claims: dynamic (atomic cursor, input order over time) or static (warp gw takes
   // chunks gw, gw + W, ...: every warp works on the same window of keys at a time)
