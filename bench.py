@@ -364,6 +364,37 @@ def main():
     stream.synchronize()
     tp_ms = ugdist.max_over_ranks(tp_s.elapsed_time(tp_e) / 1e3) * 1e3 / args.steps
 
+    # ---- host-only reference: the same kernels on just this batch's host keys ---------
+    # (how close the whole step is to the time its host rows alone take on this box; the
+    # host source is translation-bound here)
+    host_only = None
+    if args.extra and args.mode == "factored":
+        loc, _ = cache.export_placement()
+        b0 = batches[args.warmup % len(batches)]
+        hk = b0[(loc[b0] >> np.uint64(56)) == np.uint64(ws)]
+        del loc
+        if len(hk):
+            dhk = torch.from_numpy(np.ascontiguousarray(hk)).to(dev)
+            hout = torch.empty((len(hk), R), dtype=torch.uint8, device=dev)
+            hms = []
+            for i in range(args.steps + 2):
+                with torch.cuda.stream(stream):
+                    flush.fill_(i & 0xFF)
+                    torch.cuda._sleep(100_000)
+                hs, he = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                hs.record(stream)
+                cache.extract(dhk, hout, stream)
+                he.record(stream)
+                stream.synchronize()
+                if i >= 2:
+                    hms.append(hs.elapsed_time(he))
+            host_only = {"host_keys": int(len(hk)), "ms": statistics.mean(hms),
+                         "host_gbs": len(hk) * R / (statistics.mean(hms) / 1e3) / 1e9,
+                         "path": cache.last_extract_path(),
+                         "how": "extract of only the timed batch's host keys, same kernels, flush and "
+                                "spin as the timed steps"}
+            del dhk, hout
+
     # ---- parity on the full-size batch (every key, byte for byte) -------------------
     parity = None
     if not args.no_verify:
@@ -512,6 +543,8 @@ def main():
                      "frac": u_roof / (ms_per_step / 1e3),
                      "note": "source bytes scaled by the batch's unique fraction (per-source mix assumed "
                              "the same for repeats); output bytes stay n * R"}
+    if host_only:
+        host_only["step_over_host_only"] = ms_per_step / host_only["ms"]
     line = {
         "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": ws, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
@@ -539,6 +572,7 @@ def main():
                             "how": "the timed batches back to back (no L2 flush, no barrier, no per-step "
                                    "sync), device time / batches, max over ranks"},
         "duplicate_aware": dup_aware,
+        "host_only": host_only,
         "kernel_ms": {"locate_bucket": statistics.mean(loc_ms), "factored_gather": statistics.mean(gat_ms)},
         "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": n * 8,
                 "d2h_bytes_per_step": stats_bytes, "ms_per_step": statistics.mean(e2e_ms),
