@@ -151,6 +151,7 @@ struct GatherParams {
   uint64_t queue_cap;              // single pass: entries per source in `queues`
   int32_t stream_regstore;         // single pass: slots leave by warp-wide stores, not bulk copies
   int32_t stream_peer_warps;       // single pass: consumer warps per peer-dedicated CTA
+  int32_t local_sms;               // two-phase, dense host: SMs copying local rows (0 = all)
   uint32_t *qctr;                  // single pass: [2][kMaxSrc][kMaxSmId] sub-queue counts / heads
 };
 
@@ -719,6 +720,15 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
                 (uint32_t)role_ctas * kGatherWarps, lane, my_src == host_src ? p.host_rows : kRowsInFlight);
 
   }
+  }
+  // Dense host bucket: optionally only `local_sms` SMs (in chip-spreading order, after the
+  // host / peer roles) copy local rows, spreading the local burst over the host-bound step
+  // (experiment: does a gentler local stream interfere less with host translation?)
+  if (host_dense && p.local_sms > 0 && !host_cta && pos >= p.num_sms - p.local_sms) {
+    // this SM is not one of the local_sms -- fall through only if it is a dedicated SM
+  } else if (host_dense && p.local_sms > 0 && !host_cta) {
+    finish_launch(p.ctrl, p.num_src, p.n_keys, 0);
+    return;
   }
   // local group: dedicated local CTAs start here; others pad once their group drains
   // TMA bulk local copies (1 always; 2 = unless the host bucket is dense -- with a
