@@ -339,11 +339,14 @@ def main():
     # kernel pass: the same steps again with the library's own events around its launches
     # (and the fused kernel's %globaltimer phase split) for the per-kernel roofline
     cache.enable_timing(True)
+    phases = []
     for i in range(args.steps):
         step(args.warmup + i, False)
         a, b = cache.last_batch_timing()
         loc_ms.append(a)
         gat_ms.append(b)
+        if cache.last_extract_path() == "fused":
+            phases.append(cache.last_batch_phases())
     stream.synchronize()
     log("per-step gather ms: " + " ".join(f"{x:.3f}" for x in gat_ms))
     step_ms = [s.elapsed_time(e) for s, e in evs]
@@ -574,6 +577,11 @@ def main():
         "duplicate_aware": dup_aware,
         "host_only": host_only,
         "kernel_ms": {"locate_bucket": statistics.mean(loc_ms), "factored_gather": statistics.mean(gat_ms)},
+        "fused_phases_ms": ({"locate_done": statistics.mean(p[0] for p in phases),
+                             "host_ordered": statistics.mean(p[1] for p in phases),
+                             "host_copies_done": statistics.mean(p[2] for p in phases),
+                             "how": "%globaltimer stamps inside the fused kernel, ms from its start"}
+                            if phases else None),
         "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": n * 8,
                 "d2h_bytes_per_step": stats_bytes, "ms_per_step": statistics.mean(e2e_ms),
                 "path": "UGache.extract(pinned host keys -> HBM rows) + ugache_last_batch_stats "

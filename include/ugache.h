@@ -341,6 +341,13 @@ ugache_status ugache_last_batch_stats(ugache_ctx *ctx, uint64_t *per_source,
 ugache_status ugache_enable_timing(ugache_ctx *ctx, int32_t on);
 ugache_status ugache_last_batch_timing(ugache_ctx *ctx, float *ms_locate, float *ms_gather);
 
+/* Diagnostic phase split of the last fused (K1+K2) launch from the kernel's %globaltimer
+ * stamps, in ms from the kernel's start: ms[0] = grid barrier released (locate done),
+ * ms[1] = host bucket range-ordered (0 if the ordered host path did not run), ms[2] = last
+ * host-copy warp done (0 likewise).  Synchronises with the last extract.  ESTATE when the
+ * last extract was not a fused launch. */
+ugache_status ugache_last_batch_phases(ugache_ctx *ctx, float *ms);
+
 /* Number of kernel launches the last extract issued (for launch accounting). */
 ugache_status ugache_last_launch_count(const ugache_ctx *ctx, int32_t *launches);
 

@@ -50,6 +50,8 @@ struct Ctrl {
   uint32_t walk_cursor;     // input-order host walk: next key index to claim
   unsigned long long t_start;    // fused kernel: %globaltimer at CTA 0's start (ns)
   unsigned long long t_located;  // fused kernel: %globaltimer when CTA 0 leaves the grid barrier
+  unsigned long long t_ordered;  // ordered host path: host CTA 0 done ordering the host bucket
+  unsigned long long t_host_done;  // ordered host path: last host-copy warp done (atomicMax)
   // single-pass (streaming) extraction
   uint32_t qhead[kMaxSrc];  // consumer cursor of each source's queue
   uint32_t chunk_cursor;    // next key chunk to locate
@@ -515,8 +517,10 @@ __device__ __forceinline__ void host_role_sorted(const GatherParams &p, const ui
                                                  uint32_t cnt, int h, int H, uint32_t *s_tab,
                                                  uint32_t walked) {
   cnt = host_order(p, b, cnt, h, H, s_tab, walked);
+  if (h == 0 && threadIdx.x == 0) p.ctrl->t_ordered = globaltimer_ns();  // phase stamp
   if ((int)(threadIdx.x >> 5) >= p.host_warps) return;  // window control
   host_copy_ordered<kRowsInFlight>(p, cnt, threadIdx.x & 31);
+  if ((threadIdx.x & 31) == 0) atomicMax(&p.ctrl->t_host_done, globaltimer_ns());
 }
 
 // Static warp striding of W warps (this one = gw) over a bucket of cnt rows of one source,
@@ -1268,7 +1272,11 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
   __shared__ uint32_t s_base[kMaxSrc];
   constexpr uint32_t kTile = kGatherThreads * kLocateItems;
   const uint32_t ntiles = (lp.n + kTile - 1) / kTile;
-  if (blockIdx.x == 0 && threadIdx.x == 0) gp.ctrl->t_start = globaltimer_ns();
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    gp.ctrl->t_start = globaltimer_ns();
+    gp.ctrl->t_ordered = 0;
+    gp.ctrl->t_host_done = 0;  // diagnostic stamps; host copies finish >> 1 us later
+  }
   // Tiles go to CTAs in chip-spreading order; CTAs left without a tile start the input-order
   // host walk at once (the host rows of a sparse batch then overlap the locate phase, as in
   // the unfactored kernel) until every tile is located.  Keys walked here are skipped by the

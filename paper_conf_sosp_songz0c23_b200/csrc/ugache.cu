@@ -1219,6 +1219,22 @@ ugache_status ugache_last_batch_timing(ugache_ctx *ctx, float *ms_locate, float 
   return UGACHE_OK;
 }
 
+ugache_status ugache_last_batch_phases(ugache_ctx *ctx, float *ms) {
+  if (!ctx || !ms) return UGACHE_EINVAL;
+  if (!ctx->last_fused || ctx->last_launches == 0 || ctx->mode != UGACHE_MODE_FACTORED)
+    return fail(ctx, UGACHE_ESTATE, "last extract was not a fused launch");
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  UG_CUDA(ctx, cudaStreamSynchronize(ctx->last_stream));
+  ugk::Ctrl c;
+  UG_CUDA(ctx, cudaMemcpy(&c, ctx->d_ctrl, sizeof(c), cudaMemcpyDeviceToHost));
+  auto rel = [&](unsigned long long t) { return t > c.t_start ? (float)((t - c.t_start) * 1e-6) : 0.f; };
+  ms[0] = rel(c.t_located);
+  ms[1] = rel(c.t_ordered);
+  ms[2] = rel(c.t_host_done);
+  return UGACHE_OK;
+}
+
 ugache_status ugache_last_launch_count(const ugache_ctx *ctx, int32_t *launches) {
   if (!ctx || !launches) return UGACHE_EINVAL;
   *launches = ctx->last_launches;

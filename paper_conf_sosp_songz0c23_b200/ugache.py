@@ -275,6 +275,12 @@ class UGache:
               self.ctx)
         return n.value
 
+    def last_batch_phases(self):
+        """(locate done, host ordered, host copies done) in ms from the fused kernel's start."""
+        ms = (ctypes.c_float * 3)()
+        check(lib().ugache_last_batch_phases(self.ctx, ms), "ugache_last_batch_phases", self.ctx)
+        return tuple(float(x) for x in ms)
+
     def last_extract_path(self) -> str:
         """'split', 'fused', 'single_pass', 'random' or 'none' (ugache_last_extract_path)."""
         p = ctypes.c_int32()
