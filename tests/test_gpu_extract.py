@@ -693,3 +693,25 @@ def test_single_pass_register_store_retire(torch_cuda, monkeypatch, G):
             check_batch(torch_cuda, c, t, keys, N, R, G)
         for g in group:
             g.close()
+
+
+def test_fused_phase_stamps(torch_cuda):
+    """ugache_last_batch_phases: after a fused launch with a dense host bucket the stamps are
+    ordered (locate <= host ordered <= host copies done <= the launch's event time); after a
+    single-pass launch the call reports ESTATE."""
+    from paper_conf_sosp_songz0c23_b200._abi import UGacheError
+    N, R = 300_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(54).permutation(N)]
+    t, (c,) = make_group(torch_cuda, N, R, 10_000, 1, h)
+    c.enable_timing(True)
+    c.set_stream("off")
+    keys = np.random.default_rng(55).integers(0, N, 200_000)   # ~97 % host keys: dense
+    check_batch(torch_cuda, c, t, keys, N, R, 1)
+    loc_ms, gat_ms = c.last_batch_timing()
+    a, b, d = c.last_batch_phases()
+    assert 0 < a <= b <= d <= (loc_ms + gat_ms) * 1.05 + 0.01
+    c.set_stream("on")
+    check_batch(torch_cuda, c, t, keys[:5000], N, R, 1)
+    with pytest.raises(UGacheError):
+        c.last_batch_phases()
+    c.close()
