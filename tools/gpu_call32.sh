@@ -1,3 +1,3 @@
 set -x
-o=gpurun_out/r1zl; mkdir -p $o
+o=gpurun_out/r1zu; mkdir -p $o
 bash tools/gpu_round_check.sh $o
