@@ -154,6 +154,7 @@ struct GatherParams {
   int32_t stream_regstore;         // single pass: slots leave by warp-wide stores, not bulk copies
   int32_t stream_peer_warps;       // single pass: consumer warps per peer-dedicated CTA
   int32_t local_sms;               // two-phase, dense host: SMs copying local rows (0 = all)
+  int32_t stream_group;            // single pass: chunks per group with non-local rows first (<= 1 off)
   uint32_t *qctr;                  // single pass: [2][kMaxSrc][kMaxSmId] sub-queue counts / heads
 };
 
@@ -786,6 +787,7 @@ constexpr int kStreamK = 2;                          // keys per lane per chunk
 constexpr uint32_t kStreamChunk = 32u * kStreamK;    // keys per chunk (one warp)
 constexpr uint32_t kNoClaim = 0xFFFFFFFFu;
 constexpr int kStreamRegRows = 4;                    // rows per step of the register path (R > 6 KB)
+constexpr int kStreamGroupMax = 8;                   // chunks per group, non-local rows first
 
 __device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t *p) {
   uint32_t v;
@@ -995,7 +997,9 @@ __device__ __forceinline__ void stream_locs(const LocateParams &lp, const Gather
 }
 
 // Chunk c whose location entries e[] are loaded (stream_keys + stream_locs).
-template <typename KeyT>
+// PART 0: the whole chunk; 1: everything but its local rows (locate bookkeeping, queued
+// entries, inline non-local rows, keys_done); 2: only its local rows (after PART 1).
+template <typename KeyT, int PART = 0>
 __device__ __forceinline__ void stream_chunk_located(const LocateParams &lp, const GatherParams &gp, uint32_t c,
                                                      const uint64_t (&e)[kStreamK], int lane, uint64_t *s_addr,
                                                      uint32_t *s_idx, uint32_t *s_inl, StreamSlots &sl) {
@@ -1012,11 +1016,12 @@ __device__ __forceinline__ void stream_chunk_located(const LocateParams &lp, con
     if (it < (int)K && (uint32_t)lane < ck && i < n) {
       if (e[it] != ~0ull) {
         s[it] = (int)(e[it] >> UGACHE_LOC_SRC_SHIFT);
-      } else {
+      } else if (PART != 2) {
         zero_row(gp.out + (uint64_t)i * R, R);  // out-of-range key
         ++nbad;
       }
     }
+    if (PART == 2) continue;
     const int si = s[it];
     const bool inl = si >= 0 && (si == gp.local_src || (si == host_src ? gp.inline_host : gp.inline_peer));
     const int qs = (si >= 0 && !inl) ? si : -1;
@@ -1042,6 +1047,7 @@ __device__ __forceinline__ void stream_chunk_located(const LocateParams &lp, con
 #pragma unroll
   for (int pass = 0; pass < 2; ++pass) {
     const bool slow_pass = (pass == 0) != (gp.stream_host_last != 0);
+    if ((PART == 1 && !slow_pass) || (PART == 2 && slow_pass)) continue;
     if (slow_pass) slow_b = nl;
 #pragma unroll
     for (int it = 0; it < kStreamK; ++it) {
@@ -1074,7 +1080,7 @@ __device__ __forceinline__ void stream_chunk_located(const LocateParams &lp, con
   // keys_done only serves consumers (a queue is final once every key is located); with no
   // queued source in this launch nobody reads it.  A chunk that reserved queue entries
   // orders the reservations before its increment; one that reserved none needs no fence.
-  if (gp.stream_queues) {
+  if (PART != 2 && gp.stream_queues) {
     if (any_queued) {
       __threadfence();
       __syncwarp();
@@ -1223,6 +1229,45 @@ __device__ __forceinline__ void stream_body(const LocateParams &lp, const Gather
       c1 = c2;
 #pragma unroll
       for (int it = 0; it < kStreamK; ++it) e0[it] = e1[it];
+    }
+  } else if (my_src < 0 && gp.stream_group > 1 && gp.stream_k == 1) {
+    // locating warp, non-local rows first: locate a group of up to kStreamGroupMax chunks,
+    // put every non-local (host) row of the group in flight, then feed the local rows --
+    // a cold host row's latency then overlaps all of the group's local work
+    bool more = true;
+    while (more) {
+      uint32_t cs[kStreamGroupMax];
+      uint64_t es[kStreamGroupMax];
+      KeyT ks[kStreamGroupMax];
+#pragma unroll
+      for (int g = 0; g < kStreamGroupMax; ++g) {
+        const bool want = more && g < gp.stream_group;
+        cs[g] = want ? claim_chunk() : kNoClaim;
+        if (want && cs[g] >= nchunks) more = false;
+        const uint32_t i = cs[g] * (uint32_t)gp.stream_ck + lane;
+        ks[g] = (cs[g] < nchunks && (uint32_t)lane < (uint32_t)gp.stream_ck && i < n)
+                    ? static_cast<const KeyT *>(lp.keys)[i] : (KeyT)0;
+      }
+#pragma unroll
+      for (int g = 0; g < kStreamGroupMax; ++g) {
+        const uint32_t i = cs[g] * (uint32_t)gp.stream_ck + lane;
+        es[g] = (cs[g] < nchunks && (uint32_t)lane < (uint32_t)gp.stream_ck && i < n &&
+                 key_in_range<KeyT>(ks[g], lp.num_rows))
+                    ? ld_nc_u64(lp.loc + (uint64_t)ks[g])
+                    : ~0ull;
+      }
+#pragma unroll
+      for (int g = 0; g < kStreamGroupMax; ++g)
+        if (cs[g] < nchunks) {
+          const uint64_t e1[kStreamK] = {es[g]};
+          stream_chunk_located<KeyT, 1>(lp, gp, cs[g], e1, lane, s_addr, s_idx, s_inl, sl);
+        }
+#pragma unroll
+      for (int g = 0; g < kStreamGroupMax; ++g)
+        if (cs[g] < nchunks) {
+          const uint64_t e1[kStreamK] = {es[g]};
+          stream_chunk_located<KeyT, 2>(lp, gp, cs[g], e1, lane, s_addr, s_idx, s_inl, sl);
+        }
     }
   } else if (my_src < 0) {  // locating warp: chunks until none are left
     while (true) {

@@ -80,7 +80,7 @@ struct ugache_ctx {
   int inline_mask = UGACHE_INLINE_HOST;      // UGACHE_OPT_INLINE
   int stream_k = 1, stream_host_last = 0, stream_host_cap = 0, stream_static = 1, stream_nap = 100,
       stream_prefetch = 0, stream_coop = 0, stream_regstore = 0,
-      stream_peer_warps = ugk::kGatherWarps, local_sms = 0;  // single-pass env knobs
+      stream_peer_warps = ugk::kGatherWarps, local_sms = 0, stream_group = 0;  // single-pass env knobs
   int host_warps = ugk::kHostWarps;  // env UGACHE_HOST_WARPS (A0 calibration knob)
   int stage_host_io = 0;             // env UGACHE_STAGE_HOST_IO=1: stage pinned host I/O too
   std::vector<int> smids;  // sorted %smid values of the device (one per SM)
@@ -412,6 +412,8 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_STREAM_K")) ctx->stream_k = std::max(1, std::min(ugk::kStreamK, atoi(e)));
   if (const char *e = getenv("UGACHE_STREAM_HOST_LAST")) ctx->stream_host_last = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_STREAM_GROUP"))
+    ctx->stream_group = std::max(0, std::min(ugk::kStreamGroupMax, atoi(e)));
   if (const char *e = getenv("UGACHE_LOCAL_SMS")) ctx->local_sms = std::max(0, atoi(e));
   if (const char *e = getenv("UGACHE_STREAM_PEER_WARPS"))
     ctx->stream_peer_warps = std::max(1, std::min(ugk::kGatherWarps, atoi(e)));
@@ -960,6 +962,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     gp.stream_regstore = ctx->stream_regstore;
     gp.stream_peer_warps = ctx->stream_peer_warps;
     gp.local_sms = ctx->local_sms;
+    gp.stream_group = ctx->stream_group;
     gp.qctr = ctx->d_qctr;
     gp.stream_bulk = R <= ugk::kBulkWarpBytes / 2 && ctx->local_bulk != 0;
     gp.stream_k = ctx->stream_k;

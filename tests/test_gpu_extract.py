@@ -715,3 +715,24 @@ def test_fused_phase_stamps(torch_cuda):
     with pytest.raises(UGacheError):
         c.last_batch_phases()
     c.close()
+
+
+@pytest.mark.parametrize("group", ["2", "3", "8"])
+@pytest.mark.parametrize("sched", ["0", "1"])
+def test_single_pass_host_first_groups(torch_cuda, monkeypatch, group, sched):
+    """Single pass with groups of chunks whose non-local rows go first (UGACHE_STREAM_GROUP):
+    every chunk processed exactly once (static and dynamic schedules), queued peers and
+    inline host rows, ragged and tiny batches."""
+    monkeypatch.setenv("UGACHE_STREAM_GROUP", group)
+    monkeypatch.setenv("UGACHE_STREAM_STATIC", sched)
+    N, R = 200_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(56).permutation(N)]
+    for G in (1, 4):
+        t, group_ = make_group(torch_cuda, N, R, 6000, G, h)
+        c = group_[0]
+        c.set_stream("on")
+        for n in (3, 4_999, 150_001, 700_000):
+            keys = np.random.default_rng(n).integers(0, N + 2, n)
+            check_batch(torch_cuda, c, t, keys, N, R, G)
+        for g in group_:
+            g.close()
