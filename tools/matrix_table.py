@@ -1,0 +1,29 @@
+#!/usr/bin/env python3
+"""Markdown table of the bench lines in a directory (tools/config_matrix.sh)."""
+import json
+import os
+import sys
+
+d = sys.argv[1]
+rows = []
+for f in sorted(os.listdir(d)):
+    if not f.endswith(".json"):
+        continue
+    try:
+        j = json.loads(open(os.path.join(d, f)).read().strip().splitlines()[-1])
+    except Exception as e:  # noqa: BLE001
+        rows.append(f"| {f} | error: {e} |")
+        continue
+    c, r = j["config"], j["roofline"]
+    ps = j["per_source_keys"]
+    n = ps["local"] + ps["peer"] + ps["host"]
+    ab = j.get("fem_ablation") or {}
+    ho = j.get("host_only") or {}
+    rows.append("| {} | {} | {:.0%} | {} | {:.4f} | {:.0f} | {} {:.2f} | {:.2f} | {} | {} | {} |".format(
+        c["workload"], c["keys_per_batch_per_gpu"], c["cache_ratio"], r.get("path"), j["ms_per_step"], j["value"],
+        r["bound"], r["frac"], j["source_mix_roofline"]["frac"], f"{ps['host'] / n:.1%}",
+        f"{ab['random_dispatch_ms_per_step']:.4f}" if ab else "-",
+        f"{ho['ms']:.4f}" if ho else "-"))
+print("| workload | keys/batch | c | path | ms/batch | GB/s | kernel roofline | source-mix frac | host share | random dispatch ms | host keys alone ms |")
+print("|---|---|---|---|---|---|---|---|---|---|---|")
+print("\n".join(rows))
