@@ -412,6 +412,11 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_STREAM_K")) ctx->stream_k = std::max(1, std::min(ugk::kStreamK, atoi(e)));
   if (const char *e = getenv("UGACHE_STREAM_HOST_LAST")) ctx->stream_host_last = atoi(e) != 0;
+  {  // row payload L2 policy (kernels.cuh c_row_evict_first), per device
+    int ef = 0;
+    if (const char *e = getenv("UGACHE_ROW_EVICT_FIRST")) ef = atoi(e) != 0;
+    UG_CUDA(ctx, cudaMemcpyToSymbol(ugk::c_row_evict_first, &ef, sizeof(ef)));
+  }
   if (const char *e = getenv("UGACHE_STREAM_GROUP"))
     ctx->stream_group = std::max(0, std::min(ugk::kStreamGroupMax, atoi(e)));
   if (const char *e = getenv("UGACHE_LOCAL_SMS")) ctx->local_sms = std::max(0, atoi(e));
