@@ -12,8 +12,8 @@
 // Orders: 0 = batch order, 1 = 4096 ranges (the library's ordering), 2 = 32768 ranges,
 // 3 = full sort.  Copy: warps of the active CTAs claim U consecutive entries from a global
 // cursor (the library's host_copy_ordered).  Active CTAs are chosen by %smid, spread over
-// the chip (every (S/H)-th SM id in ascending order).  Also: the copy engine via
-// cudaMemcpyBatchAsync of 512-B copies, for the same rows.
+// the chip (every (S/H)-th SM id in ascending order).  (An earlier copy-engine leg with one
+// 512-B copy per row was removed: that batched-copy call is closed on this GPU pool.)
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <sys/mman.h>
@@ -259,38 +259,6 @@ int main(int argc, char **argv) {
           fflush(stdout);
         }
       }
-    }
-    // copy engine: one 512-B cudaMemcpyBatchAsync op per row, same order
-    if (!quick) {
-      std::vector<void *> dsts(n), srcs(n);
-      std::vector<size_t> sizes(n, R);
-      for (uint32_t i = 0; i < n; ++i) {
-        dsts[i] = out + (size_t)i * R;
-        srcs[i] = h + (size_t)rows[i] * R;
-      }
-      cudaMemcpyAttributes attr = {};
-      attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-      attr.flags = cudaMemcpyFlagPreferOverlapWithCompute;
-      size_t idx0 = 0, fail = 0;
-      float best = 1e9;
-      cudaStream_t st;
-      CK(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
-      for (int rep = 0; rep < 3; ++rep) {
-        cudaEventRecord(a, st);
-        cudaError_t e = cudaMemcpyBatchAsync(dsts.data(), srcs.data(), sizes.data(), n, &attr, &idx0, 1, &fail, st);
-        cudaEventRecord(b, st);
-        if (e != cudaSuccess) {
-          fprintf(stderr, "cudaMemcpyBatchAsync: %s (fail idx %zu)\n", cudaGetErrorString(e), fail);
-          cudaGetLastError();
-          break;
-        }
-        CK(cudaEventSynchronize(b));
-        float ms;
-        cudaEventElapsedTime(&ms, a, b);
-        best = std::min(best, ms);
-      }
-      printf("%d,ce,0,0,%.4f,%.2f\n", order, best, (double)n * R / (best * 1e-3) / 1e9);
-      CK(cudaStreamDestroy(st));
     }
   }
   // sequential reference: rows 0..n-1
