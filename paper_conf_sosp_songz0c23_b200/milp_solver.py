@@ -50,84 +50,102 @@ def make_blocks(h_sorted: np.ndarray, G: int, max_frac: float = 0.005) -> List[T
 
 def solve_blocks(h_sorted: np.ndarray, blocks, C: int, G: int, T, Rr, time_limit: float = 60.0):
     """Block MILP.  T = (T_local, T_peer, T_host), Rr = (R_local, R_peer, R_host).
-    Returns (s[G, B] bool, a[G, G+1, B] bool, z seconds, status message)."""
+    Returns (s[G, B] bool, a[G, G+1, B] bool, z seconds, status message).
+
+    The model is assembled block-major with numpy index arrays: every constraint family is
+    one vectorised batch of rows of a COO matrix.  Column layout, with M = G + 1 sources
+    (source G = host) and times in units of T_local for conditioning:
+
+      s[b, j]      B*G    binary   block b stored on GPU j
+      a[b, i, j]   B*G*M  binary   GPU i reads block b from source j
+      u[i, j]      G*M    >= 0     t^j_i, modeled time of GPU i's reads from j
+      t[i]         G      >= 0     t_i
+      z            1      >= 0     objective
+    """
     import scipy.sparse as sp
     from scipy.optimize import Bounds, LinearConstraint, milp
 
-    B = len(blocks)
-    M = G + 1
+    B, M = len(blocks), G + 1
     hs = np.maximum(np.asarray(h_sorted, dtype=np.float64), 0.0)
-    mass = np.array([hs[a:b].sum() for a, b in blocks])
-    size = np.array([b - a for a, b in blocks], dtype=np.float64)
-    scale = T[0] if T[0] > 0 else 1.0
+    cum = np.concatenate([[0.0], np.cumsum(hs)])
+    lo_r = np.array([a for a, _ in blocks], dtype=np.int64)
+    hi_r = np.array([b for _, b in blocks], dtype=np.int64)
+    mass = cum[hi_r] - cum[lo_r]                       # H_b: hotness mass of block b
+    size = (hi_r - lo_r).astype(np.float64)            # n_b: entries of block b
+    unit = T[0] if T[0] > 0 else 1.0
+    # T[i, j] and R[i, j]: peer everywhere, local on the diagonal, host in the last column
+    Tm = np.full((G, M), T[1] / unit)
+    Rm = np.full((G, M), float(Rr[1]))
+    Tm[np.arange(G), np.arange(G)] = T[0] / unit
+    Rm[np.arange(G), np.arange(G)] = Rr[0]
+    Tm[:, G] = T[2] / unit
+    Rm[:, G] = Rr[2]
 
-    def Trow(i):
-        t = np.full(M, T[1]) / scale
-        t[i] = T[0] / scale
-        t[G] = T[2] / scale
-        return t
+    n_s, n_a, n_u = B * G, B * G * M, G * M
+    S = np.arange(n_s).reshape(B, G)
+    A = n_s + np.arange(n_a).reshape(B, G, M)
+    U = n_s + n_a + np.arange(n_u).reshape(G, M)
+    Tt = n_s + n_a + n_u + np.arange(G)
+    Z = n_s + n_a + n_u + G
+    nv = Z + 1
 
-    def Rrow(i):
-        r = np.full(M, Rr[1])
-        r[i] = Rr[0]
-        r[G] = Rr[2]
-        return r
-
-    ia = lambda i, j, b: (i * M + j) * B + b
-    na = G * M * B
-    is_ = lambda j, b: na + j * B + b
-    ns = G * B
-    itj = lambda i, j: na + ns + i * M + j
-    it = lambda i: na + ns + G * M + i
-    iz = na + ns + G * M + G
-    nv = iz + 1
     rows, cols, vals, lo, hi = [], [], [], [], []
-    r = [0]
+    nrow = 0
 
-    def add(ent, l, u):
-        for c, v in ent:
-            rows.append(r[0])
-            cols.append(c)
-            vals.append(v)
-        lo.append(l)
-        hi.append(u)
-        r[0] += 1
+    def family(r_idx, c_idx, v, l, u, count):
+        """count constraint rows; entry k sits in row r_idx[k] (relative) at column c_idx[k]."""
+        nonlocal nrow
+        rows.append(np.asarray(r_idx, dtype=np.int64).ravel() + nrow)
+        cols.append(np.asarray(c_idx, dtype=np.int64).ravel())
+        vals.append(np.broadcast_to(np.asarray(v, dtype=np.float64), np.shape(c_idx)).ravel())
+        lo.append(np.broadcast_to(np.float64(l), (count,)))
+        hi.append(np.broadcast_to(np.float64(u), (count,)))
+        nrow += count
 
-    for i in range(G):
-        for b in range(B):
-            add([(ia(i, j, b), 1.0) for j in range(M)], 1.0, 1.0)
-    for i in range(G):
-        for j in range(G):
-            for b in range(B):
-                add([(is_(j, b), 1.0), (ia(i, j, b), -1.0)], 0.0, np.inf)
-    for j in range(G):
-        add([(is_(j, b), size[b]) for b in range(B)], -np.inf, float(C))
-    for i in range(G):
-        Ti = Trow(i)
-        for j in range(M):
-            add([(itj(i, j), 1.0)] + [(ia(i, j, b), -Ti[j] * mass[b]) for b in range(B)], 0.0, 0.0)
-    for i in range(G):
-        for j in range(M):
-            add([(it(i), 1.0), (itj(i, j), -1.0)], 0.0, np.inf)
-        Ri = Rrow(i)
-        add([(it(i), 1.0)] + [(itj(i, j), -Ri[j]) for j in range(M)], 0.0, np.inf)
-        add([(iz, 1.0), (it(i), -1.0)], 0.0, np.inf)
-    A = sp.csr_array((vals, (rows, cols)), shape=(r[0], nv))
+    # every GPU reads every block from exactly one source:  sum_j a[b,i,j] = 1
+    r = np.broadcast_to(np.arange(B * G).reshape(B, G, 1), (B, G, M))
+    family(r, A, 1.0, 1.0, 1.0, B * G)
+    # a GPU source must store what is read from it:  s[b,j] - a[b,i,j] >= 0  (j < G)
+    r = np.arange(B * G * G).reshape(B, G, G)
+    family(np.stack([r, r], -1), np.stack([np.broadcast_to(S[:, None, :], (B, G, G)), A[:, :, :G]], -1),
+           np.array([1.0, -1.0]), 0.0, np.inf, B * G * G)
+    # capacity, counted in entries (block sizes):  sum_b n_b s[b,j] <= C
+    family(np.broadcast_to(np.arange(G), (B, G)), S, np.broadcast_to(size[:, None], (B, G)),
+           -np.inf, float(C), G)
+    # u[i,j] = T[i,j] * sum_b H_b a[b,i,j]
+    r_u = np.arange(G * M).reshape(G, M)
+    family(np.concatenate([r_u.ravel(), np.broadcast_to(r_u, (B, G, M)).ravel()]),
+           np.concatenate([U.ravel(), A.ravel()]),
+           np.concatenate([np.ones(G * M), (-Tm[None, :, :] * mass[:, None, None]).ravel()]),
+           0.0, 0.0, G * M)
+    # t_i >= u[i,j]
+    family(np.stack([r_u, r_u], -1), np.stack([np.broadcast_to(Tt[:, None], (G, M)), U], -1),
+           np.array([1.0, -1.0]), 0.0, np.inf, G * M)
+    # t_i >= sum_j R[i,j] u[i,j]
+    family(np.concatenate([np.arange(G), np.repeat(np.arange(G), M)]),
+           np.concatenate([Tt, U.ravel()]), np.concatenate([np.ones(G), -Rm.ravel()]),
+           0.0, np.inf, G)
+    # z >= t_i
+    family(np.stack([np.arange(G)] * 2, -1), np.stack([np.full(G, Z), Tt], -1),
+           np.array([1.0, -1.0]), 0.0, np.inf, G)
+
+    Am = sp.coo_array((np.concatenate(vals), (np.concatenate(rows), np.concatenate(cols))),
+                      shape=(nrow, nv)).tocsr()
     c = np.zeros(nv)
-    c[iz] = 1.0
-    integ = np.zeros(nv)
-    integ[: na + ns] = 1
+    c[Z] = 1.0
+    binary = np.zeros(nv)
+    binary[: n_s + n_a] = 1
     ub = np.full(nv, np.inf)
-    ub[: na + ns] = 1.0
-    res = milp(c, integrality=integ, bounds=Bounds(np.zeros(nv), ub),
-               constraints=LinearConstraint(A, lo, hi),
+    ub[: n_s + n_a] = 1.0
+    res = milp(c, integrality=binary, bounds=Bounds(np.zeros(nv), ub),
+               constraints=LinearConstraint(Am, np.concatenate(lo), np.concatenate(hi)),
                options=dict(time_limit=time_limit, disp=False, mip_rel_gap=1e-6))
     if res.x is None:
         raise RuntimeError(f"block MILP failed: {res.message}")
     x = res.x
-    s = np.array([[x[is_(j, b)] > 0.5 for b in range(B)] for j in range(G)])
-    a = np.array([[[x[ia(i, j, b)] > 0.5 for b in range(B)] for j in range(M)] for i in range(G)])
-    return s, a, float(x[iz]) * scale, res.message
+    s_out = (x[S] > 0.5).T                              # [G, B]
+    a_out = np.transpose(x[A] > 0.5, (1, 2, 0))         # [G, M, B]
+    return s_out, a_out, float(x[Z]) * unit, res.message
 
 
 def placement_from_blocks(order: np.ndarray, blocks, s: np.ndarray, a: np.ndarray, N: int, G: int):

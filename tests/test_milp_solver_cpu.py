@@ -1,7 +1,9 @@
 """CPU tests of the block-level MILP solver (paper_conf_sosp_songz0c23_b200/milp_solver.py,
-section 6.3): block construction rules, agreement with the entry-level MILP oracle when
-blocks are single entries, and consistency of the produced placement with the oracle's
-section 6.2 model and placement checker."""
+section 6.3): block construction rules; the solver's optimum against an independent
+brute-force enumeration of block placements (multi-entry blocks, size-weighted capacity);
+agreement with the entry-level MILP oracle when blocks are single entries; and consistency
+of the produced placement with the oracle's section 6.2 model and placement checker."""
+import itertools
 import math
 
 import numpy as np
@@ -75,3 +77,66 @@ def test_block_placement_is_valid_and_matches_model(G, E, C):
     z_part = sweep_z(h, order, E, C, _plat(G), 0)
     # block granularity can cost a little against entry-level policies (paper: < 2 %)
     assert z <= min(z_rep, z_part) * 1.02
+
+
+def _block_brute_force(mass, size, C, G, T, Rr):
+    """Exact optimum of the block model by enumeration, independent of any MILP: every
+    storage choice (a subset of blocks per GPU, sum of its block sizes <= C), and for each
+    GPU every access arrangement over the sources that hold the block (or the host).  Per
+    block b and GPU i the sources are 0..G-1 (GPU j; j == i local) and G (host); a GPU's time
+    is max(max_j t^j_i, sum_j R_{i<-j} t^j_i) with t^j_i = T_{i<-j} * (mass read from j)
+    (P:1359-1385), and z = max over GPUs.  Returns (z, storage masks)."""
+    B = len(mass)
+    srcs = G + 1
+    acc = np.array(list(itertools.product(range(srcs), repeat=B)), dtype=np.int64)  # [K, B]
+    bits = 1 << np.arange(B)
+    need = np.stack([((acc == j) * bits).sum(axis=1) for j in range(G)], axis=1)    # [K, G]
+    t_gpu = []
+    for i in range(G):
+        Ti = np.array([T[0] if j == i else (T[2] if j == G else T[1]) for j in range(srcs)])
+        Ri = np.array([Rr[0] if j == i else (Rr[2] if j == G else Rr[1]) for j in range(srcs)])
+        per_src = np.stack([((acc == j) * mass).sum(axis=1) * Ti[j] for j in range(srcs)], axis=1)
+        t_gpu.append(np.maximum(per_src.max(axis=1), per_src @ Ri))                # [K]
+    sizes = np.array([sum(size[b] for b in range(B) if m >> b & 1) for m in range(1 << B)])
+    fits = [m for m in range(1 << B) if sizes[m] <= C]
+    best, arg = np.inf, None
+    for stores in itertools.product(fits, repeat=G):
+        st = np.array(stores)
+        ok = (need & ~st[None, :]) == 0                                            # [K, G]
+        feasible = ok.all(axis=1)
+        z = max(t_gpu[i][feasible].min() for i in range(G))
+        if z < best:
+            best, arg = z, stores
+    return best, arg
+
+
+@pytest.mark.parametrize("G,sizes,C,seed", [
+    (2, [3, 1, 2, 4, 2, 5], 6, 0),     # multi-entry blocks, capacity binds mid-block
+    (2, [2, 2, 2, 2, 2, 2], 5, 1),
+    (2, [1, 4, 1, 3, 2], 4, 2),
+    (3, [2, 3, 1, 2], 4, 3),
+])
+def test_block_milp_equals_brute_force(G, sizes, C, seed):
+    """Independent pin of solve_blocks (not derived from oracle/milp.py): on multi-entry blocks
+    its objective equals the exact optimum found by enumerating every block storage (size-
+    weighted capacity) and access arrangement, and its own storage/access realise that value
+    under the oracle's entry-level model (oracle.placement.model_times)."""
+    rng = np.random.default_rng(seed)
+    E = int(sum(sizes))
+    blocks, b0 = [], 0
+    for sz in sizes:
+        blocks.append((b0, b0 + sz))
+        b0 += sz
+    h = np.sort(rng.pareto(1.2, E).astype(np.float32) + 0.05)[::-1].copy()   # sorted hotness
+    plat = Platform(G=G, row_bytes=512, host_sms=8, peer_sms=(148 - 8) // (G - 1), **B200)
+    T, Rr = plat.T(), plat.ratios()
+    mass = np.array([h[a:b].astype(np.float64).sum() for a, b in blocks])
+    z_bf, _ = _block_brute_force(mass, np.array(sizes), C, G, T, Rr)
+    s, a, z, _ = solve_blocks(h, blocks, C, G, T, Rr)
+    assert abs(z - z_bf) <= 1e-6 * z_bf, (z, z_bf)
+    assert all(sum(sizes[b] for b in range(len(sizes)) if s[j, b]) <= C for j in range(G))
+    order = np.arange(E)                                # h is already in rank order
+    locs, sks = placement_from_blocks(order, blocks, s, a, E, G)
+    check_placement(np.stack(locs), sks, E, C, local_preference=False)
+    zm, _, _ = model_times(h, np.stack(locs), plat)
+    assert abs(zm - z) <= 1e-6 * z
