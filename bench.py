@@ -34,6 +34,43 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 
 METRIC = "extraction GB/s (n*R/t_batch, all GPUs), ms/batch, % of source-mix roofline"
+NVLINK_GBS = 770.0   # B200_PROFILING.md: measured peer copy per direction
+
+
+def batch_roofline(P, n, R, kb, path, hbm, pcie, nvl):
+    """Source-mix roofline of one batch on every GPU.
+
+    P[g, j]: keys GPU g read from source j in the batch (j = g local, j < G peer, j = G host);
+    n[g]: keys of GPU g's batch; R: row bytes; kb: key bytes; path: the extract path taken;
+    hbm / nvl: GB/s; pcie[g]: GB/s of GPU g's host link.  Per GPU, algorithmic bytes:
+      HBM      n_L*R (local reads) + n*R (out writes) + n*(kb + 8) (keys + location entries)
+               + bucket traffic (16 B/key two-phase; 16 B per queued peer key single pass)
+               + B_served (rows the peers read from this GPU's slab)
+      NVLink   ingress sum_j n_Pj*R; egress B_served
+      PCIe     n_H*R
+    T_roof(g) = max of the four terms / their bandwidths; the batch roofline is max over g.
+    Also the bytes of the timed kernel alone ("kernel_bytes": the split path times K2 only,
+    whose HBM bytes are n_L*R + n*R + 8n bucket reads + B_served)."""
+    P = np.asarray(P, dtype=np.float64)
+    G = P.shape[0]
+    served = P[:, :G].sum(axis=0) - np.diag(P[:, :G])          # rows read from g by peers
+    ranks = []
+    for g in range(G):
+        n_l, n_h = P[g, g], P[g, G]
+        n_p = P[g, :G].sum() - n_l
+        bucket = 16.0 * (n_p if path == "single_pass" else n[g])
+        b = {"hbm": n_l * R + n[g] * R + n[g] * (kb + 8) + bucket + served[g] * R,
+             "pcie": n_h * R, "nvlink_in": n_p * R, "nvlink_out": served[g] * R}
+        kbytes = dict(b)
+        if path == "split":
+            kbytes["hbm"] = n_l * R + n[g] * R + 8.0 * n[g] + served[g] * R
+        bw = {"hbm": hbm, "pcie": pcie[g], "nvlink_in": nvl, "nvlink_out": nvl}
+        t = {k: (b[k] / (bw[k] * 1e9) if bw[k] else 0.0) for k in b}
+        kt = {k: (kbytes[k] / (bw[k] * 1e9) if bw[k] else 0.0) for k in b}
+        ranks.append({"bytes": b, "t_s": t, "t_roof_s": max(t.values()), "bound": max(t, key=t.get),
+                      "kernel_bytes": kbytes, "kernel_bound": max(kt, key=kt.get)})
+    bounding = int(np.argmax([r["t_roof_s"] for r in ranks]))
+    return {"ranks": ranks, "t_roof_s": ranks[bounding]["t_roof_s"], "bounding_rank": bounding}
 
 
 def log(*a):
@@ -68,7 +105,56 @@ def parse():
     ap.add_argument("--extra", dest="extra", action="store_true", default=True,
                     help="also time the random-dispatch (unfactored) ablation (default)")
     ap.add_argument("--no-extra", dest="extra", action="store_false")
+    ap.add_argument("--share-gpus", action="store_true",
+                    help="allow more ranks than visible GPUs (functional multi-rank runs on one "
+                         "GPU; gloo control plane); otherwise that is an error")
+    ap.add_argument("--alias-gb", type=float, default=0.0,
+                    help="full-size key span on a smaller box: back the N-row host table with this "
+                         "many GB of physical rows mapped repeatedly (synth.AliasedHostTable); the "
+                         "host tier is then off (it would need the full span physically)")
+    ap.add_argument("--print-world", action="store_true",
+                    help="print this rank's RANK/WORLD_SIZE as JSON and exit (launch check)")
     return ap.parse_args()
+
+
+def _free_port() -> int:
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def launch_ranks(args):
+    """--gpus N (N > 1) needs N ranks, one per GPU.  Under torchrun WORLD_SIZE must equal N
+    (else exit 2).  Without a torchrun environment, re-run this very command under
+    torch.distributed.run with N local ranks (127.0.0.1 rendezvous) and exit with its status,
+    so `python bench.py --gpus N` never silently measures one GPU."""
+    ws_env = os.environ.get("WORLD_SIZE")
+    if ws_env is not None:
+        if int(ws_env) != args.gpus and args.impl != "reference":
+            log(f"error: --gpus {args.gpus} but WORLD_SIZE {ws_env}")
+            sys.exit(2)
+        return
+    if args.gpus <= 1 or args.impl == "reference":
+        return
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={args.gpus}", "--master-addr", "127.0.0.1",
+           "--master-port", str(_free_port()), os.path.abspath(__file__)] + sys.argv[1:]
+    log("launching " + " ".join(cmd[1:]))
+    sys.exit(subprocess.run(cmd).returncode)
+
+
+def shm_plan(bytes_needed: int, path: str = "/dev/shm"):
+    """(ok, free bytes) of the shared-memory filesystem that holds the node's host table and
+    host tier at N > 1."""
+    try:
+        st = os.statvfs(path)
+        free = st.f_bavail * st.f_frsize
+    except OSError:
+        return False, 0
+    return bytes_needed <= free, free
 
 
 def dist_env():
@@ -145,9 +231,29 @@ def pcie_h2d_peak(torch) -> float:
     return n / (best * 1e-3) / 1e9
 
 
-def setup_table(wl, rank, ws, torch_dist):
+def mem_available() -> int:
+    try:
+        with open("/proc/meminfo") as f:
+            for line in f:
+                if line.startswith("MemAvailable:"):
+                    return int(line.split()[1]) * 1024
+    except OSError:
+        pass
+    return 0
+
+
+def setup_table(wl, rank, ws, torch_dist, alias_gb=0.0):
     import synth
     t0 = time.time()
+    if alias_gb > 0 and wl.table_bytes > alias_gb * 1e9:
+        if ws > 1:
+            raise SystemExit("--alias-gb is single-process only")
+        table = synth.AliasedHostTable(wl.num_rows, wl.row_bytes, int(alias_gb * 1e9) // wl.row_bytes)
+        table.fill()
+        log(f"aliased table: {wl.num_rows} rows x {wl.row_bytes} B span ({wl.table_bytes / 1e9:.1f} GB) "
+            f"backed by {table.phys_rows} physical rows ({table.phys_bytes / 1e9:.1f} GB) mapped "
+            f"{table.copies} times, in {time.time() - t0:.1f}s")
+        return table
     if ws == 1:
         table = synth.HostTable(wl.num_rows, wl.row_bytes)
         table.fill()
@@ -179,8 +285,16 @@ def run_reference(args, wl):
     if rank != 0:
         return
     import synth
-    table = synth.HostTable(wl.num_rows, wl.row_bytes)
-    table.fill()
+    avail = mem_available()
+    if args.alias_gb > 0 and wl.table_bytes > args.alias_gb * 1e9:
+        table = setup_table(wl, 0, 1, None, args.alias_gb)
+    elif avail and wl.table_bytes > 0.9 * avail:
+        print(json.dumps({"impl": "reference", "unavailable": f"the {wl.table_bytes / 1e9:.0f} GB table does "
+                          f"not fit host RAM; rerun with --alias-gb"}), flush=True)
+        return
+    else:
+        table = synth.HostTable(wl.num_rows, wl.row_bytes)
+        table.fill()
     batches = make_batches(wl, 0, max(1, min(args.batches, args.steps)))
     n = len(batches[0])
     out = np.empty((n, wl.row_bytes), dtype=np.uint8)
@@ -214,6 +328,9 @@ def config_dict(args, wl, ws):
             "alpha": wl.alpha, "cache_ratio": args.cache_ratio if args.cache_ratio is not None
             else wl.cache_ratio, "policy": args.policy, "mode": args.mode, "stream": args.stream, "inline": args.inline,
             "host_tier": bool(getattr(args, "host_tier", False)),
+            "host_table": (f"aliased: {args.alias_gb:g} GB of physical rows mapped over the full "
+                           f"{wl.table_bytes / 1e9:.0f} GB span" if getattr(args, "alias_gb", 0) and
+                           wl.table_bytes > args.alias_gb * 1e9 else "full"),
             "parallelism": f"dp{ws}",
             "l2": "256 MiB L2-flush write between timed steps (outside the events); per-step "
                   "output > L2",
@@ -223,6 +340,12 @@ def config_dict(args, wl, ws):
 
 def main():
     args = parse()
+    launch_ranks(args)
+    if args.print_world:
+        rank, ws, local = dist_env()
+        print(json.dumps({"rank": rank, "world_size": ws, "local_rank": local, "gpus": args.gpus}),
+              flush=True)
+        return
     import synth
     wl = synth.get_workload(args.workload)
     if args.cache_ratio is not None:
@@ -237,9 +360,25 @@ def main():
     import oracle
     from paper_conf_sosp_songz0c23_b200 import UGache, dist as ugdist, make_config, solve
     rank, ws, local = dist_env()
-    if ws != args.gpus:
-        log(f"warning: --gpus {args.gpus} but WORLD_SIZE {ws}; using WORLD_SIZE")
     ndev = torch.cuda.device_count()
+    if ndev < 1:
+        log("error: no CUDA device visible")
+        sys.exit(3)
+    if ws > ndev and not args.share_gpus:
+        log(f"error: {ws} ranks but only {ndev} GPUs visible (use --share-gpus for a functional "
+            f"multi-rank run on shared GPUs)")
+        sys.exit(3)
+    if ws > 1:
+        # the node's host table (+ tier) live in /dev/shm, shared by the ranks
+        need = wl.table_bytes * (2 if args.host_tier else 1)
+        ok, free = shm_plan(need)
+        if not ok and args.host_tier and shm_plan(wl.table_bytes)[0]:
+            log(f"/dev/shm has {free / 1e9:.1f} GB free < table + tier {need / 1e9:.1f} GB: "
+                f"running without the shared host tier")
+            args.host_tier = False
+        elif not ok:
+            log(f"error: /dev/shm has {free / 1e9:.1f} GB free < host table {wl.table_bytes / 1e9:.1f} GB")
+            sys.exit(4)
     dev_idx = local % ndev
     torch.cuda.set_device(dev_idx)
     dev = torch.device("cuda", dev_idx)
@@ -252,7 +391,16 @@ def main():
             tdist.init_process_group("gloo")
     local = dev_idx
 
-    table = setup_table(wl, rank, ws, tdist)
+    aliased = args.alias_gb > 0 and wl.table_bytes > args.alias_gb * 1e9
+    avail = mem_available()
+    if ws == 1 and not aliased and avail and wl.table_bytes > 0.9 * avail:
+        log(f"error: the {wl.table_bytes / 1e9:.0f} GB table does not fit the {avail / 1e9:.0f} GB of "
+            f"available host RAM; use --alias-gb or a row-scaled workload (name@scale)")
+        sys.exit(4)
+    if args.host_tier and (aliased or (ws == 1 and avail and 2 * wl.table_bytes > 0.85 * avail)):
+        log("host tier off: it needs another full copy of the table in host RAM")
+        args.host_tier = False
+    table = setup_table(wl, rank, ws, tdist, args.alias_gb)
     t0 = time.time()
     h = synth.hotness(wl)
     log(f"hotness in {time.time() - t0:.1f}s")
@@ -350,6 +498,8 @@ def main():
     stream.synchronize()
     log("per-step gather ms: " + " ".join(f"{x:.3f}" for x in gat_ms))
     step_ms = [s.elapsed_time(e) for s, e in evs]
+    # a multi-GPU step lasts as long as its slowest rank: per-step max over ranks
+    step_max = ugdist.gather_rows(step_ms).max(axis=0)
     my_total_s = sum(step_ms) / 1e3
     max_total_s = ugdist.max_over_ranks(my_total_s)
     bytes_all = ugdist.sum_over_ranks(float(args.steps * n * R))
@@ -481,67 +631,62 @@ def main():
     peaks = measured_peaks()
     hbm = float(peaks.get("hbm_gbs", 6650.0))
     hbm_src = "MEASURED_PEAKS.json hbm_gbs" if "hbm_gbs" in peaks else "B200_PROFILING.md fallback"
-    pcie = pcie_h2d_peak(torch) if rank == 0 else 0.0
-    per = np.mean(np.stack(per_src), axis=0)
-    G = ws
-    n_local = float(per[rank]) if G > 0 else 0.0
-    n_host = float(per[G])
-    n_peer = float(per.sum() - n_local - n_host)
+    # PCIe reference measured on every rank at once (all local GPUs reading host memory
+    # concurrently, as during the timed steps): each rank's own pinned-H2D copy rate
+    ugdist.barrier()
+    pcie = pcie_h2d_peak(torch)
+    nvl = NVLINK_GBS
     kb = 8 if dkeys[0].dtype == torch.int64 else 4
-    # the timed kernel: K2 alone (two launches) or the whole fused K1+K2 launch
-    kern_ms = [a + b for a, b in zip(loc_ms, gat_ms)] if launches == args.steps else list(gat_ms)
-    gat_s = statistics.mean(kern_ms) / 1e3
-    loc_s = statistics.mean(loc_ms) / 1e3
-    # algorithmic bytes of the timed kernel: rows read per source + rows
-    # written + key + location entry per key, plus the bucket traffic of the path taken:
-    #   fused K1+K2 (one launch): 16 B/key (bucket write + read);
-    #   split: K2 alone is timed (8 B/key bucket read; K1 is its own launch);
-    #   single pass K3: no local bucket -- only queued (peer) rows take 16 B
     path = statistics.mode(paths)
+    # the timed kernel: K2 alone (two launches) or the whole fused / single-pass launch
+    kern_ms = [a + b for a, b in zip(loc_ms, gat_ms)] if launches == args.steps else list(gat_ms)
+    per = np.mean(np.stack(per_src), axis=0)
+    # every rank's numbers, so the batch roofline is the max over GPUs
+    mine = np.concatenate([per.astype(np.float64),
+                           [n, statistics.mean(kern_ms), statistics.mean(loc_ms), statistics.mean(step_ms),
+                            pcie, tp_ms]])
+    allr = ugdist.gather_rows(mine)
+    P = allr[:, :ws + 1]
+    n_all = allr[:, ws + 1]
+    kern_all, loc_all, step_all, pcie_all = allr[:, ws + 2], allr[:, ws + 3], allr[:, ws + 4], allr[:, ws + 5]
+    rl = batch_roofline(P, n_all, R, kb, path, hbm, pcie_all, nvl)
+    slow = int(np.argmax(kern_all))            # the rank whose kernel sets the batch time
+    kr = rl["ranks"][slow]
+    bound = kr["kernel_bound"]
+    kbytes = kr["kernel_bytes"][bound]
+    peak = {"hbm": hbm, "pcie": pcie_all[slow], "nvlink_in": nvl, "nvlink_out": nvl}[bound]
+    psrc = {"hbm": hbm_src,
+            "pcie": "live cudaMemcpy pinned H2D 1 GiB best-of-5 on every rank at once, this run",
+            "nvlink_in": "B200_PROFILING.md measured peer copy",
+            "nvlink_out": "B200_PROFILING.md measured peer copy"}[bound]
+    gat_s = kern_all[slow] / 1e3
+    achieved = kbytes / gat_s / 1e9
+    unit = "GB/s"
     kname = {"single_pass": "stream_extract_kernel", "fused": "fused_extract_kernel"}.get(
         path, "factored_gather_kernel")
-    fused = path in ("fused", "single_pass")
-    k1_hbm_bytes = n * (kb + 8 + 8)
-    if path == "single_pass":
-        gather_hbm_bytes = n_local * R + n * R + n * (kb + 8) + n_peer * 16
-    else:
-        gather_hbm_bytes = n_local * R + n * R + n * 8 + (k1_hbm_bytes if fused else 0)
-    gather_pcie_bytes = n_host * R
-    t_hbm = gather_hbm_bytes / (hbm * 1e9)
-    t_pcie = gather_pcie_bytes / (pcie * 1e9) if pcie else 0.0
-    nvl = 770.0
-    t_nvl = n_peer * R / (nvl * 1e9)
-    terms = {"hbm": t_hbm, "pcie": t_pcie, "nvlink": t_nvl}
-    bound = max(terms, key=terms.get)
-    if bound == "hbm":
-        achieved, peak, unit, psrc = gather_hbm_bytes / gat_s / 1e9, hbm, "GB/s", hbm_src
-    elif bound == "pcie":
-        achieved, peak, unit, psrc = gather_pcie_bytes / gat_s / 1e9, pcie, "GB/s", \
-            "live cudaMemcpy pinned H2D 1 GiB best-of-5 in this run"
-    else:
-        achieved, peak, unit, psrc = n_peer * R / gat_s / 1e9, nvl, "GB/s", \
-            "B200_PROFILING.md measured peer copy"
-    # whole-step source-mix roofline (locate + gather): every byte the step moves
-    step_hbm = gather_hbm_bytes if path == "single_pass" else n_local * R + n * R + n * 8 + k1_hbm_bytes
-    t_roof = max(step_hbm / (hbm * 1e9), t_pcie, t_nvl)
-    ms_per_step = statistics.mean(step_ms)
+    n_local, n_host = float(per[rank]), float(per[ws])
+    n_peer = float(per.sum() - n_local - n_host)
+    ms_per_step = float(np.mean(step_max))
+    t_roof = rl["t_roof_s"]
     traffic = traffic_pcie = traffic_src = None
-    try:  # per-launch DRAM traffic of K2 from the committed ncu capture of this workload
+    try:  # per-launch DRAM traffic of the kernel from the committed ncu capture of this config
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
             rec = json.load(f)[wl.name][kname]
         c_run = args.cache_ratio if args.cache_ratio is not None else wl.cache_ratio
-        if abs(rec.get("cache_ratio", wl.cache_ratio) - c_run) < 1e-9:  # same workload only
+        if (abs(rec.get("cache_ratio", wl.cache_ratio) - c_run) < 1e-9 and
+                bool(rec.get("host_tier", False)) == bool(args.host_tier) and rec.get("n_gpus", 1) == ws):
             traffic, traffic_pcie, traffic_src = rec["dram_bytes"], rec.get("pcie_read_bytes"), rec["source"]
     except Exception:
         pass
     # duplicate-aware variant: source reads counted per unique row of the
-    # batch (repeats are L2 hits), against the same bandwidths
+    # batch (repeats are L2 hits), against the same bandwidths (this rank's batch)
     uniq = len(np.unique(batches[args.warmup % len(batches)]))
     dup_aware = None
     if uniq < n:
         fu = uniq / n
+        mr = rl["ranks"][rank]
         u_hbm = n_local * fu * R + n * R + n * (kb + 8) + (16 * n if path != "single_pass" else n_peer * 16)
-        u_roof = max(u_hbm / (hbm * 1e9), (t_pcie * fu), t_nvl * fu)
+        u_roof = max(u_hbm / (hbm * 1e9), mr["t_s"]["pcie"] * fu, mr["t_s"]["nvlink_in"] * fu)
         dup_aware = {"unique_keys": uniq, "unique_frac": fu, "t_roof_us": u_roof * 1e6,
                      "frac": u_roof / (ms_per_step / 1e3),
                      "note": "source bytes scaled by the batch's unique fraction (per-source mix assumed "
@@ -553,33 +698,46 @@ def main():
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
         "config": config_dict(args, wl, ws),
-        "roofline": {"bound": bound, "achieved": achieved, "peak": peak, "unit": unit,
+        "roofline": {"bound": "pcie" if bound == "pcie" else ("hbm" if bound == "hbm" else "nvlink"),
+                     "term": bound, "achieved": achieved, "peak": peak, "unit": unit,
                      "frac": achieved / peak if peak else None, "traffic": traffic,
                      "traffic_pcie_read": traffic_pcie, "traffic_source": traffic_src,
-                     "algorithmic_bytes": {"hbm": gather_hbm_bytes, "pcie": gather_pcie_bytes,
-                                           "nvlink": n_peer * R},
+                     "algorithmic_bytes": kr["kernel_bytes"],
                      "kernel": kname + {"fused": " (K1 locate+bucket and K2 gather, one cooperative launch)",
                                         "single_pass": " (K3: locate + copy in one pass, no grid barrier)"}.get(path, ""),
-                     "path": path,
+                     "path": path, "rank": slow,
                      "peak_source": psrc,
-                     "kernel_ms": statistics.mean(kern_ms)},
+                     "kernel_ms": kern_all[slow],
+                     "how": "algorithmic bytes of the kernel's bounding term on the rank with the longest "
+                            "kernel time, / that rank's mean kernel time (CUDA events on the extract stream)"},
         "source_mix_roofline": {"t_roof_us": t_roof * 1e6, "t_step_us": ms_per_step * 1e3,
                                 "frac": t_roof / (ms_per_step / 1e3),
-                                "terms_us": {"hbm": step_hbm / (hbm * 1e9) * 1e6,
-                                             "pcie": t_pcie * 1e6, "nvlink": t_nvl * 1e6},
-                                "bw_gbs": {"hbm": hbm, "pcie": pcie, "nvlink": nvl}},
+                                "bounding_rank": rl["bounding_rank"],
+                                "terms_us": {k: v * 1e6 for k, v in rl["ranks"][rl["bounding_rank"]]["t_s"].items()},
+                                "bw_gbs": {"hbm": hbm, "pcie": float(np.min(pcie_all)), "nvlink": nvl},
+                                "how": "T_roof = max over GPUs g of max(HBM bytes incl. rows served to peers "
+                                       "/ BW_HBM, NVLink ingress / BW_NVL, NVLink egress (rows peers read "
+                                       "from g) / BW_NVL, host rows / BW_PCIe(g)); t_step = mean over steps "
+                                       "of the max over ranks"},
         "per_source_keys": {"local": n_local, "peer": n_peer, "host": n_host},
-        "ms_p50": float(np.percentile(step_ms, 50)), "ms_p99": float(np.percentile(step_ms, 99)),
+        "per_rank": ({"keys_from_source": P.tolist(), "kernel_ms": kern_all.tolist(),
+                      "step_ms": step_all.tolist(), "pcie_peak_gbs": pcie_all.tolist(),
+                      "t_roof_us": [r_["t_roof_s"] * 1e6 for r_ in rl["ranks"]]} if ws > 1 else None),
+        "ms_p50": float(np.percentile(step_max, 50)), "ms_p99": float(np.percentile(step_max, 99)),
         "throughput_mode": {"ms_per_batch": tp_ms, "value": ugdist.sum_over_ranks(float(n * R)) / (tp_ms / 1e3) / 1e9,
                             "unit": "GB/s",
                             "how": "the timed batches back to back (no L2 flush, no barrier, no per-step "
                                    "sync), device time / batches, max over ranks"},
         "duplicate_aware": dup_aware,
         "host_only": host_only,
-        "kernel_ms": {"locate_bucket": statistics.mean(loc_ms), "factored_gather": statistics.mean(gat_ms)},
+        "kernel_ms": {"locate_bucket": float(np.max(loc_all)),
+                      "factored_gather": float(np.max(kern_all - (loc_all if launches == args.steps else 0))),
+                      "how": "max over ranks of each rank's mean"},
         "fused_phases_ms": ({"locate_done": statistics.mean(p[0] for p in phases),
                              "host_ordered": statistics.mean(p[1] for p in phases),
                              "host_copies_done": statistics.mean(p[2] for p in phases),
+                             "last_cta_located": statistics.mean(p[3] for p in phases),
+                             "launch_end": statistics.mean(p[4] for p in phases),
                              "how": "%globaltimer stamps inside the fused kernel, ms from its start"}
                             if phases else None),
         "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": n * 8,
@@ -595,7 +753,7 @@ def main():
                 "staged_readback": {"value": e2e_staged_value,
                                     "ms_per_step": statistics.mean(e2e_staged_ms),
                                     "path": "H2D keys + extract + D2H rows (cudaMemcpyAsync)"}},
-        "gpu_launches": launches,
+        "gpu_launches": int(ugdist.sum_over_ranks(float(launches))),
         "clocks": clk,
         "parity": parity,
         "plan": {"k": plan.k, "band_end": plan.band_end, "capacity_rows": plan.capacity_rows,
@@ -628,7 +786,7 @@ def main():
     cache.close()
     ugdist.barrier()
     for buf in (table, tier):
-        if isinstance(buf, synth.HostTable):
+        if isinstance(buf, (synth.HostTable, synth.AliasedHostTable)):
             path = buf.shm_path
             buf.close()
             if ws > 1 and rank == 0 and path and os.path.exists(path):

@@ -92,7 +92,8 @@ typedef struct {
  * ranks >= band_end) are read from a pinned host copy laid out in hotness-rank order
  * instead of the caller's key-ordered table, so host reads concentrate in a dense prefix
  * of host address space.  Location-table rows of the host source are then tier slots
- * (slot t holds the key of rank band_end + t) instead of keys. */
+ * (slot t holds the key of rank (band_end + t) mod N) instead of keys; the tier holds all N
+ * rows so that a cache refresh can redirect any evicted key to it. */
 #define UGACHE_FLAG_HOST_TIER 1
 
 /* Solver output (section 6.2 model evaluated for the chosen placement). */
@@ -108,6 +109,11 @@ typedef struct {
   double T_local, T_peer, T_host;  /* T_{i<-j} per entry (s)               */
   double R_local, R_peer, R_host;  /* R_{i<-j} core ratios                   */
   int32_t host_sms, peer_sms, num_sms, reserved;
+  double host_mass_frac;   /* hotness mass of the host-resident ranks (>= band_end) over the
+                              total: the expected host share of a batch's keys (hotness =
+                              expected accesses per batch, R6).  The extract path
+                              choice uses it until this ctx has run a launch.  0 = unknown
+                              (ugache_init_with_placement).                                */
 } ugache_plan;
 
 /* ---- host-only placement solver (no GPU needed) ------------------------------------ */
@@ -127,11 +133,13 @@ ugache_status ugache_build_placement(const ugache_config *cfg, const uint64_t *o
                                      const ugache_plan *plan, int32_t gpu, uint64_t *loc,
                                      uint64_t *slot_keys, uint64_t *n_slots);
 
-/* Host tier (UGACHE_FLAG_HOST_TIER): number of tier rows, N - band_end. */
+/* Host tier (UGACHE_FLAG_HOST_TIER): number of tier rows -- N: the tier holds every row in
+ * hotness-rank order rotated so the host-resident ranks [band_end, N) come first (slot t =
+ * rank (band_end + t) mod N); the cached ranks' slots serve keys a refresh evicts. */
 uint64_t ugache_host_tier_rows(const ugache_plan *plan, uint64_t num_rows);
 
-/* Fill a caller-provided host tier: tier[t*R ..) = table row order[band_end + t] for
- * t < tier_rows (parallel host copy, no GPU).  tier: ugache_host_tier_rows * R bytes. */
+/* Fill a caller-provided host tier: tier[t*R ..) = table row order[(band_end + t) mod N]
+ * for t < N (parallel host copy, no GPU).  tier: ugache_host_tier_rows * R bytes. */
 ugache_status ugache_fill_host_tier(const ugache_config *cfg, const uint64_t *order,
                                     const ugache_plan *plan, const void *host_table,
                                     void *tier);
@@ -140,15 +148,17 @@ ugache_status ugache_fill_host_tier(const ugache_config *cfg, const uint64_t *or
 
 /* Create the ctx of GPU cfg->rank on device cfg->device: solve the placement, build this
  * GPU's location table in HBM, allocate the cache slab (C x R bytes, its own cudaMalloc so
- * it can be IPC-exported) and the bucket scratch.  host_table: N*R bytes, caller-owned, must
- * outlive the ctx and stay unmodified (read-only access); it is page-locked and
+ * it can be IPC-exported) and the bucket scratch.  host_table: N*R bytes, 16-byte aligned
+ * (else EINVAL), caller-owned, must outlive the ctx and stay unmodified (read-only access); it is page-locked and
  * mapped with cudaHostRegister unless already pinned.  hotness: as for ugache_solve,
  * copied.  The cache is NOT filled: call ugache_fill, connect peers, then barrier. */
 ugache_status ugache_init(ugache_ctx **ctx, const ugache_config *cfg, const void *host_table,
                           const float *hotness);
 
 /* Same as ugache_init but with a precomputed order/plan (every rank of a process group can
- * share one solve).  order: N entries; plan from ugache_solve with the same cfg.
+ * share one solve).  order: N entries, a permutation of [0, N) (else EINVAL); plan from
+ * ugache_solve with the same cfg (its capacity_rows <= min(C, N), k <= capacity_rows <=
+ * band_end <= N, and the same SM dedication, else EINVAL).
  * host_tier: with UGACHE_FLAG_HOST_TIER, an optional caller-owned tier already filled by
  * ugache_fill_host_tier (shared by the ranks of a node; pinned by the library unless
  * already pinned; must outlive the ctx); NULL = the ctx builds and owns its own tier.
@@ -183,7 +193,8 @@ ugache_status ugache_ipc_handle(ugache_ctx *ctx, void *buf, size_t *len);
 ugache_status ugache_open_peers(ugache_ctx *ctx, const void *all_handles, size_t len_each);
 
 /* In-process alternative to IPC: slabs[j] = device address of GPU j's slab, reachable from
- * this ctx's device (same device, or peer access enabled).  slabs[rank] is ignored. */
+ * this ctx's device (same device, or peer access enabled), 16-byte aligned.  slabs[rank] is
+ * ignored. */
 ugache_status ugache_set_peer_slabs(ugache_ctx *ctx, const void *const *slabs);
 
 /* Filler: copy this GPU's cached rows from the host table into its slab
@@ -192,7 +203,8 @@ ugache_status ugache_set_peer_slabs(ugache_ctx *ctx, const void *const *slabs);
 ugache_status ugache_fill(ugache_ctx *ctx, void *stream);
 
 /* THE HOT PATH.  out[i*R .. (i+1)*R) = table row keys[i] for i < n (output in
- * key order P:626-627).  keys: n keys of key_type, device or host memory.  out: n*R bytes,
+ * key order P:626-627).  keys: n keys of key_type, device or host memory, aligned to the
+ * key size (else EINVAL).  out: n*R bytes,
  * device or host memory, 16-byte aligned.  Device buffers: fully asynchronous on stream,
  * no host synchronisation, no collective; keys/out must stay valid until the stream
  * reaches the work.  Pinned (page-locked) host buffers: read / written in place by the
@@ -232,25 +244,86 @@ ugache_status ugache_msg_scatter(ugache_ctx *ctx, const void *replies, void *out
 /* ---- cache refresh (section 7.2) ----------------------------------------
  * "Refresher evicts old entries and inserts new entries into UGache's hashtable and cache
  * content ... Refresher waits for a foreground batch between the update of hashtable and
- * cache content".  Three calls per GPU; between them the CALLER makes every
- * GPU of the group reach the same step and lets one foreground batch finish:
- *   1. ugache_refresh_begin(new placement): every key whose location changes is pointed at
- *      the host now (async on stream); extracts stay correct and simply read those keys
- *      from host DRAM.   -> all GPUs, then >= 1 foreground batch + barrier
- *   2. ugache_refresh_content(max_sms, max_rows, &remaining): rewrite the slots whose key
- *      changes from the host table (only those), at most max_rows per call (0 = all) with
- *      at most max_sms SMs' worth of CTAs (0 = all) -- the refresh granularity / resource
- *      throttle of P:1611-1616; synchronous; call again while remaining > 0 (foreground
- *      batches may run in between).   -> all GPUs, then barrier
- *   3. ugache_refresh_commit: install the new location table and slot list.
- * new_loc / new_slot_keys: as for ugache_init_with_placement (checked the same way).  Not
- * available with UGACHE_FLAG_HOST_TIER.  Wrong order -> ESTATE. */
+ * cache content".  new_loc / new_slot_keys: as for ugache_init_with_placement
+ * (checked the same way; host rows = keys -- with UGACHE_FLAG_HOST_TIER the library maps
+ * them to tier slots, the tier holding every row).  Every call below is asynchronous on
+ * stream except where noted; between steps the CALLER makes every GPU of the group reach
+ * the same step (barrier) and, where stated, lets one foreground batch finish.  Wrong
+ * order -> ESTATE.
+ *
+ * Whole-table protocol (three calls per GPU):
+ *   1. ugache_refresh_begin(new placement): stage it (synchronises stream; uploads the new
+ *      table), then every key whose location changes is pointed at the host (which holds
+ *      every entry); extracts stay correct and read those keys from host DRAM.
+ *      -> all GPUs, then >= 1 foreground batch + barrier
+ *   2. ugache_refresh_content(max_sms, max_rows, &remaining): rewrite the next max_rows
+ *      (0 = all) slots whose key changes from the host table with at most max_sms SMs'
+ *      worth of CTAs (0 = all) -- the refresh granularity / resource throttle of
+ *      P:1611-1616; call again while remaining > 0.  -> all GPUs: synchronise the stream,
+ *      then barrier
+ *   3. ugache_refresh_commit: install the new location table and slot list (synchronises).
+ *
+ * Chunked protocol (the incremental refill of SURVEY.md 8(f) row 3): only one slot range is
+ * in transition at a time, so at most that chunk's keys are redirected to the host.
+ *   ugache_refresh_stage(new placement)                 (synchronous; no table change)
+ *   for each slot range [lo, hi) covering [0, capacity_rows), on every GPU:
+ *     ugache_refresh_chunk(EVICT, lo, hi): keys whose current location is a GPU slot in
+ *        [lo, hi) and changes -> host.   -> all GPUs, >= 1 foreground batch + barrier
+ *     ugache_refresh_chunk(FILL, lo, hi, max_sms): rewrite this GPU's changed slots in
+ *        [lo, hi).   -> all GPUs: synchronise the stream, then barrier
+ *     ugache_refresh_chunk(INSTALL, lo, hi): keys whose new location is a GPU slot in
+ *        [lo, hi) take it.
+ *   ugache_refresh_commit                                (synchronous) */
+enum { UGACHE_REFRESH_EVICT = 0, UGACHE_REFRESH_FILL = 1, UGACHE_REFRESH_INSTALL = 2 };
 ugache_status ugache_refresh_begin(ugache_ctx *ctx, const uint64_t *new_loc,
                                    const uint64_t *new_slot_keys, uint64_t n_new_slots,
                                    void *stream);
 ugache_status ugache_refresh_content(ugache_ctx *ctx, int32_t max_sms, uint64_t max_rows,
                                      uint64_t *remaining, void *stream);
+ugache_status ugache_refresh_stage(ugache_ctx *ctx, const uint64_t *new_loc,
+                                   const uint64_t *new_slot_keys, uint64_t n_new_slots,
+                                   void *stream);
+ugache_status ugache_refresh_chunk(ugache_ctx *ctx, int32_t step, uint64_t slot_lo,
+                                   uint64_t slot_hi, int32_t max_sms, void *stream);
 ugache_status ugache_refresh_commit(ugache_ctx *ctx, void *stream);
+
+/* Section 6.2 model value z (seconds) of a given placement under hotness (P:1359-1385,
+ * P:1497-1498): locs[i] = GPU i's location table (N entries, UGACHE_LOC_* encoding; only
+ * the source field is used), hotness = N floats (NULL = uniform; <= 0 counts as 0; NaN/Inf
+ * -> EINVAL), T_{i<-j} / R_{i<-j} from plan.  The Refresher's trigger compares the current
+ * placement's z under fresh hotness with a new solve's z.  Host-only. */
+ugache_status ugache_model_time(const ugache_plan *plan, int32_t num_gpus, uint64_t num_rows,
+                                const uint64_t *const *locs, const float *hotness, double *z);
+
+/* ---- A0 calibration (Fig. 6; section 5.3) -------------------
+ * Bandwidth vs the number of SMs dedicated to a source, measured through this ctx's own
+ * sources with the extract kernels' SM placement (roles spread over the chip): the host
+ * source (tier or table: sorted uniform random rows, the range-ordered host reads), every
+ * peer at once (k SMs per peer, all-to-all ingress), and the local slab (all SMs).  L2 is
+ * flushed before every timed launch.  "Realistic contention": call it on every
+ * rank of the group at the same time (caller barrier before), so the host link and each
+ * GPU's NVLink egress carry the load of all G readers.  Synchronous (uses the legacy
+ * stream and a temporary 256 MiB device buffer).  Results (reading R13 of DESIGN.md):
+ *   host_sms = the smallest swept SM count reaching >= 90 % of the best host bandwidth;
+ *   bw_host  = the bandwidth at host_sms (bytes/s of row payload);
+ *   peer_sms = the same rule on the aggregate peer ingress with k SMs per peer, capped at
+ *              floor((S - host_sms) / (G - 1)) (0 when G == 1 or peers are not connected);
+ *   bw_peer  = aggregate ingress at peer_sms (the ugache_config bw_peer unit);
+ *   bw_local = local random-row gather with every SM (bytes/s of rows read).
+ * The curves are returned point by point.  Requires ugache_fill (and peers when G > 1). */
+#define UGACHE_CALIB_MAX_POINTS 24
+typedef struct {
+  int32_t host_sms, peer_sms;
+  double bw_local, bw_peer, bw_host;
+  int32_t n_host_points, n_peer_points;
+  int32_t host_points_sms[UGACHE_CALIB_MAX_POINTS];
+  double host_points_bw[UGACHE_CALIB_MAX_POINTS];
+  int32_t peer_points_sms[UGACHE_CALIB_MAX_POINTS];
+  double peer_points_bw[UGACHE_CALIB_MAX_POINTS];
+  uint32_t sample_rows;      /* rows per source per timed launch */
+  int32_t reserved;
+} ugache_calibration;
+ugache_status ugache_calibrate(ugache_ctx *ctx, uint32_t sample_rows, ugache_calibration *out);
 
 /* Core dedication override: SMs for host and for each peer; local gets the
  * rest plus padding.  0 keeps the current value.  Only affects later extracts. */
@@ -290,8 +363,15 @@ typedef enum {
   UGACHE_OPT_LOCAL_BULK = 8,
   UGACHE_OPT_EARLY_WALK = 9,
   UGACHE_OPT_STREAM = 10,
-  UGACHE_OPT_INLINE = 11
+  UGACHE_OPT_INLINE = 11,
+  UGACHE_OPT_PREORDER = 12
 } ugache_option;
+/* UGACHE_OPT_PREORDER (default 1): on the two-phase paths (fused / split) with host
+ *   ordering on, the locate pass counts each host entry into its key-range histogram, and
+ *   right after the locate | gather boundary every CTA of the launch scans the histogram
+ *   and scatters its slice of the host bucket into range order; the host-copy warps start
+ *   as soon as all CTAs are done.  0 = the host CTAs alone order the bucket after the
+ *   boundary (histogram | barrier | scan | scatter | barrier).  Same output bytes. */
 /* UGACHE_OPT_STREAM: single-pass extraction (K3, its own cooperative kernel).  Warps take
  *   64-key chunks (a static schedule: warp w takes chunks w, w + W, ...), locate them (A1)
  *   and copy local rows at once (A4: local extraction tolerates every core);
@@ -342,10 +422,12 @@ ugache_status ugache_enable_timing(ugache_ctx *ctx, int32_t on);
 ugache_status ugache_last_batch_timing(ugache_ctx *ctx, float *ms_locate, float *ms_gather);
 
 /* Diagnostic phase split of the last fused (K1+K2) launch from the kernel's %globaltimer
- * stamps, in ms from the kernel's start: ms[0] = grid barrier released (locate done),
- * ms[1] = host bucket range-ordered (0 if the ordered host path did not run), ms[2] = last
- * host-copy warp done (0 likewise).  Synchronises with the last extract.  ESTATE when the
- * last extract was not a fused launch. */
+ * stamps, in ms from the kernel's start (CTA 0's first instruction): ms[0] = grid barrier
+ * released (locate done), ms[1] = host bucket range-ordered (0 if the ordered host path
+ * did not run), ms[2] = last host-copy warp done (0 likewise), ms[3] = the last CTA
+ * finished its locate tiles, ms[4] = the last CTA of the launch finished.  ms: 5 floats.
+ * Synchronises with the last extract.  ESTATE when the last extract was not a fused
+ * launch. */
 ugache_status ugache_last_batch_phases(ugache_ctx *ctx, float *ms);
 
 /* Number of kernel launches the last extract issued (for launch accounting). */

@@ -10,7 +10,7 @@ The product is ``libugache.so`` (C ABI in ``include/ugache.h``, sm_100a kernels 
 * :mod:`.build`  -- nvcc build of the library (sm_100a).
 """
 from .ugache import (UGache, build_placement, connect_in_process, fill_host_tier,  # noqa: F401
-                     host_tier_rows, make_config, solve)
+                     host_tier_rows, make_config, model_time, solve)
 
 __all__ = ["UGache", "solve", "build_placement", "make_config", "connect_in_process",
-           "fill_host_tier", "host_tier_rows"]
+           "fill_host_tier", "host_tier_rows", "model_time"]

@@ -26,8 +26,9 @@ KEY_I64, KEY_U32 = 0, 1
 MODE_FACTORED, MODE_RANDOM_DISPATCH = 0, 1
 OPT_HOST_ORDERING, OPT_STAGE_HOST_IO, OPT_HOST_WARPS = 0, 1, 2
 OPT_DEDICATION, OPT_WARP_HOST, OPT_WARP_PEER, OPT_HOST_WALK, OPT_FUSED = 3, 4, 5, 6, 7
-OPT_LOCAL_BULK, OPT_EARLY_WALK, OPT_STREAM, OPT_INLINE = 8, 9, 10, 11
+OPT_LOCAL_BULK, OPT_EARLY_WALK, OPT_STREAM, OPT_INLINE, OPT_PREORDER = 8, 9, 10, 11, 12
 INLINE_HOST, INLINE_PEERS = 1, 2
+REFRESH_EVICT, REFRESH_FILL, REFRESH_INSTALL = 0, 1, 2
 PATHS = {0: "none", 1: "split", 2: "fused", 3: "single_pass", 4: "random"}
 DEDICATE_SMS, DEDICATE_WARPS = 0, 1
 FLAG_HOST_TIER = 1
@@ -53,10 +54,26 @@ class ugache_plan(ctypes.Structure):
                 ("T_host", ctypes.c_double), ("R_local", ctypes.c_double),
                 ("R_peer", ctypes.c_double), ("R_host", ctypes.c_double),
                 ("host_sms", ctypes.c_int32), ("peer_sms", ctypes.c_int32),
-                ("num_sms", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("num_sms", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("host_mass_frac", ctypes.c_double)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_ if f != "reserved"}
+
+
+CALIB_MAX_POINTS = 24
+
+
+class ugache_calibration(ctypes.Structure):
+    _fields_ = [("host_sms", ctypes.c_int32), ("peer_sms", ctypes.c_int32),
+                ("bw_local", ctypes.c_double), ("bw_peer", ctypes.c_double),
+                ("bw_host", ctypes.c_double), ("n_host_points", ctypes.c_int32),
+                ("n_peer_points", ctypes.c_int32),
+                ("host_points_sms", ctypes.c_int32 * CALIB_MAX_POINTS),
+                ("host_points_bw", ctypes.c_double * CALIB_MAX_POINTS),
+                ("peer_points_sms", ctypes.c_int32 * CALIB_MAX_POINTS),
+                ("peer_points_bw", ctypes.c_double * CALIB_MAX_POINTS),
+                ("sample_rows", ctypes.c_uint32), ("reserved", ctypes.c_int32)]
 
 
 _c = ctypes
@@ -90,6 +107,11 @@ SIGNATURES = {
     "ugache_refresh_begin": (_ST, [_P, _P, _P, _c.c_uint64, _P]),
     "ugache_refresh_content": (_ST, [_P, _c.c_int32, _c.c_uint64, ctypes.POINTER(_c.c_uint64), _P]),
     "ugache_refresh_commit": (_ST, [_P, _P]),
+    "ugache_calibrate": (_ST, [_P, _c.c_uint32, ctypes.POINTER(ugache_calibration)]),
+    "ugache_refresh_stage": (_ST, [_P, _P, _P, _c.c_uint64, _P]),
+    "ugache_refresh_chunk": (_ST, [_P, _c.c_int32, _c.c_uint64, _c.c_uint64, _c.c_int32, _P]),
+    "ugache_model_time": (_ST, [ctypes.POINTER(ugache_plan), _c.c_int32, _c.c_uint64, _P, _P,
+                                ctypes.POINTER(_c.c_double)]),
     "ugache_set_dedication": (_ST, [_P, _c.c_int32, _c.c_int32]),
     "ugache_set_mode": (_ST, [_P, _c.c_int32]),
     "ugache_set_option": (_ST, [_P, _c.c_int32, _c.c_int64]),

@@ -46,6 +46,7 @@ struct Ctrl {
   uint32_t stat_bad;
   uint32_t host_arrive[2];  // intra-role barriers of the host CTAs
   uint32_t host_cursor;     // dynamic cursor over the range-ordered host bucket
+  uint32_t host_seg_cursor[8];  // per-segment cursors (host_segments > 1)
   uint32_t grid_arrive;     // grid barrier of the fused locate+gather kernel
   uint32_t walk_cursor;     // input-order host walk: next key index to claim
   unsigned long long t_start;    // fused kernel: %globaltimer at CTA 0's start (ns)
@@ -58,6 +59,12 @@ struct Ctrl {
   uint32_t keys_done;       // keys whose chunk is fully located (queued or copied)
   uint32_t stat_n;          // keys of the last launch (auto mode: previous batch's host density)
   uint32_t last_stream;     // 1 = the last launch ran the single-pass path
+  // host pre-ordering (range histogram built during locate): CTAs done scattering their
+  // slice of the host bucket into range order
+  uint32_t pre_arrive;
+  unsigned long long t_loc_max;   // latest %globaltimer at which a CTA finished its locate tiles
+  unsigned long long t_loc_last;  // t_loc_max of the last launch (published by finish_launch)
+  unsigned long long t_end;       // %globaltimer when the last CTA of the last launch finished
   // pinned, device-mapped host words {n, host count, launches} written by the last CTA of
   // every launch: the host picks the next batch's path from them without synchronising
   volatile uint32_t *host_mirror;
@@ -94,6 +101,10 @@ struct LocateParams {
   uint32_t n;
   uint32_t row_bytes;
   int32_t num_src;
+  // host pre-ordering: histogram of the host rows' key ranges, built while locating
+  int32_t hist;              // 1 = count every host entry into range_count
+  uint32_t range_shift;      // range = row >> range_shift
+  uint32_t *range_count;     // kMaxRanges counters, zero between launches
 };
 
 struct GatherParams {
@@ -156,6 +167,12 @@ struct GatherParams {
   int32_t local_sms;               // two-phase, dense host: SMs copying local rows (0 = all)
   int32_t stream_group;            // single pass: chunks per group with non-local rows first (<= 1 off)
   uint32_t *qctr;                  // single pass: [2][kMaxSrc][kMaxSmId] sub-queue counts / heads
+  int32_t preorder;                // the locate pass built the host range histogram: every CTA
+                                   // scatters a slice of the host bucket (preorder_host)
+  int32_t hist_smem;               // fused kernel: the histogram is aggregated per CTA in shared
+                                   // memory before the global atomics
+  int32_t host_segments;           // ordered host copy: the ordered bucket is split into this many
+                                   // segments read concurrently (1 = one cursor, in order)
 };
 
 struct RandomParams {
@@ -284,8 +301,13 @@ __device__ __forceinline__ void finish_launch(Ctrl *ctrl, int num_src, uint32_t 
       c->host_arrive[0] = 0;
       c->host_arrive[1] = 0;
       c->host_cursor = 0;
+      for (int k = 0; k < 8; ++k) c->host_seg_cursor[k] = 0;
       c->grid_arrive = 0;
       c->walk_cursor = 0;
+      c->pre_arrive = 0;
+      c->t_loc_last = c->t_loc_max;
+      c->t_loc_max = 0;
+      c->t_end = globaltimer_ns();
       __threadfence();
       c->done = 0;
     }
@@ -297,7 +319,8 @@ __device__ __forceinline__ void finish_launch(Ctrl *ctrl, int num_src, uint32_t 
 // shared arrays of kMaxSrc entries; the function starts and ends with a CTA barrier.
 template <typename KeyT, int THREADS>
 __device__ __forceinline__ void locate_tile(const LocateParams &p, uint64_t tile,
-                                            uint32_t *s_cnt, uint32_t *s_base) {
+                                            uint32_t *s_cnt, uint32_t *s_base,
+                                            uint32_t *s_hist = nullptr) {
   const int tid = threadIdx.x, lane = tid & 31;
   __syncthreads();
   if (tid < kMaxSrc) s_cnt[tid] = 0;
@@ -353,6 +376,8 @@ __device__ __forceinline__ void locate_tile(const LocateParams &p, uint64_t tile
       const uint32_t row = (uint32_t)(e[it] & UGACHE_LOC_ROW_MASK);
       p.buckets[(uint64_t)src[it] * p.bucket_cap + s_base[src[it]] + pos[it]] =
           ((uint64_t)row << 32) | (uint64_t)i;
+      if (p.hist && src[it] == p.num_src - 1)
+        atomicAdd(s_hist ? &s_hist[row >> p.range_shift] : &p.range_count[row >> p.range_shift], 1u);
     }
   }
 }
@@ -433,8 +458,26 @@ __device__ __forceinline__ void block_exclusive_scan(const uint32_t *src, uint32
 // In-order copy of the range-ordered host bucket: warps claim U consecutive entries from a
 // shared cursor (next claim prefetched), so the rows in flight are the most recent claims.
 template <int U>
-__device__ __forceinline__ void host_copy_ordered(const GatherParams &p, uint32_t cnt, int lane) {
+__device__ __forceinline__ void host_copy_ordered(const GatherParams &p, uint32_t cnt, int lane,
+                                                  uint32_t gwarp) {
   const uint8_t *base = p.base[p.num_src - 1];
+  const int K = min(max(p.host_segments, 1), 8);
+  if (K > 1) {
+    // K contiguous segments of the ordered bucket read at once (warp w starts on segment
+    // w mod K, then helps the others): the rows in flight mix dense and sparse key ranges
+    for (int t = 0; t < K; ++t) {
+      const uint32_t sg = (gwarp + (uint32_t)t) % (uint32_t)K;
+      const uint32_t lo = (uint32_t)((uint64_t)cnt * sg / K), hi = (uint32_t)((uint64_t)cnt * (sg + 1) / K);
+      while (true) {
+        uint32_t e0 = 0;
+        if (lane == 0) e0 = lo + atomicAdd(&p.ctrl->host_seg_cursor[sg], (uint32_t)U);
+        e0 = __shfl_sync(kFullMask, e0, 0);
+        if (e0 >= hi) break;
+        copy_rows<U>(base, p.out, p.row_bytes, p.host_sorted + e0, (int)min((uint32_t)U, hi - e0), lane);
+      }
+    }
+    return;
+  }
   uint32_t next = 0;
   if (lane == 0) next = atomicAdd(&p.ctrl->host_cursor, (uint32_t)U);
   next = __shfl_sync(kFullMask, next, 0);
@@ -482,6 +525,49 @@ __device__ __forceinline__ uint32_t host_order(const GatherParams &p, const uint
     }
   }
   return total;
+}
+
+// Range ordering without the host CTAs' serial prefix (gp.preorder): the locate pass already
+// counted every host entry into range_count, so right after the locate | gather boundary
+// EVERY CTA of the launch scans the counts (4096 entries, on-chip) and scatters its
+// 1/gridDim slice of the host bucket into range order, then arrives on pre_arrive.  The
+// host-copy warps start once all CTAs arrived (host_role_preordered) -- a few microseconds
+// instead of the host CTAs' histogram | barrier | scan | scatter | barrier sequence.  With a
+// sparse host bucket the histogram is unused and each CTA re-arms its slice of it.
+__device__ __forceinline__ void preorder_host(const GatherParams &p, uint32_t *s_tab, uint32_t pos,
+                                              uint32_t S) {
+  const int tid = threadIdx.x;
+  const int host_src = p.num_src - 1;
+  const uint32_t cnt = *(volatile const uint32_t *)&p.ctrl->counts[host_src];
+  if (cnt < p.host_sort_min) {
+    const uint32_t zlo = p.n_ranges * pos / S, zhi = p.n_ranges * (pos + 1) / S;
+    for (uint32_t i = zlo + tid; i < zhi; i += blockDim.x) p.range_count[i] = 0;
+    return;
+  }
+  block_exclusive_scan(p.range_count, s_tab, p.n_ranges);
+  const uint64_t *b = p.buckets + (uint64_t)host_src * p.bucket_cap;
+  const uint32_t lo = (uint32_t)((uint64_t)cnt * pos / S), hi = (uint32_t)((uint64_t)cnt * (pos + 1) / S);
+  for (uint32_t e = lo + tid; e < hi; e += blockDim.x) {
+    const uint64_t ent = b[e];
+    const uint32_t r = (uint32_t)(ent >> 32) >> p.range_shift;
+    p.host_sorted[s_tab[r] + atomicAdd(&p.range_cursor[r], 1u)] = ent;
+  }
+  __syncthreads();
+  if (tid == 0) {
+    __threadfence();
+    atomicAdd(&p.ctrl->pre_arrive, 1u);
+  }
+}
+
+// After preorder_host: wait until every CTA scattered its slice, then re-arm slice h of H of
+// the range counters (every CTA has read range_count and bumped range_cursor by now).
+__device__ __forceinline__ void preorder_wait(const GatherParams &p, uint32_t h, uint32_t H) {
+  role_wait(&p.ctrl->pre_arrive, gridDim.x);
+  const uint32_t zlo = p.n_ranges * h / H, zhi = p.n_ranges * (h + 1) / H;
+  for (uint32_t i = zlo + threadIdx.x; i < zhi; i += blockDim.x) {
+    p.range_count[i] = 0;
+    p.range_cursor[i] = 0;
+  }
 }
 
 // Input-order host walk (sparse host buckets, and the fused kernel's early walk): warps
@@ -533,10 +619,11 @@ __device__ __forceinline__ void host_walk_copy(const GatherParams &p, int warp, 
 __device__ __forceinline__ void host_role_sorted(const GatherParams &p, const uint64_t *b,
                                                  uint32_t cnt, int h, int H, uint32_t *s_tab,
                                                  uint32_t walked) {
-  cnt = host_order(p, b, cnt, h, H, s_tab, walked);
+  if (p.preorder) preorder_wait(p, (uint32_t)h, (uint32_t)H);  // ordered by every CTA already
+  else cnt = host_order(p, b, cnt, h, H, s_tab, walked);
   if (h == 0 && threadIdx.x == 0) p.ctrl->t_ordered = globaltimer_ns();  // phase stamp
   if ((int)(threadIdx.x >> 5) >= p.host_warps) return;  // window control
-  host_copy_ordered<kRowsInFlight>(p, cnt, threadIdx.x & 31);
+  host_copy_ordered<kRowsInFlight>(p, cnt, threadIdx.x & 31, (uint32_t)(h * p.host_warps) + (threadIdx.x >> 5));
   if ((threadIdx.x & 31) == 0) atomicMax(&p.ctrl->t_host_done, globaltimer_ns());
 }
 
@@ -684,6 +771,7 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
   asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
   const int pos = smid < (uint32_t)kMaxSmId ? p.sm_pos[smid] : p.num_sms - 1;
   const int host_src = p.num_src - 1;
+  if (p.preorder) preorder_host(p, s_dyn, blockIdx.x, gridDim.x);
   const uint32_t n_host = p.ctrl->counts[host_src];
   const bool host_dense = p.host_sort && n_host >= p.host_sort_min;
   const uint32_t R = p.row_bytes;
@@ -698,9 +786,15 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
     // and no SM idles behind a slow link.
     const int S = p.num_sms, hw = p.host_warps, pw = p.peer_warps;
     const uint64_t *bh = p.buckets + (uint64_t)host_src * p.bucket_cap;
-    const uint32_t n_ord = host_dense ? host_order(p, bh, n_host, pos, S, s_dyn, 0) : 0;
+    uint32_t n_ord = 0;
+    if (host_dense && p.preorder) {
+      preorder_wait(p, blockIdx.x, gridDim.x);
+      n_ord = n_host;
+    } else if (host_dense) {
+      n_ord = host_order(p, bh, n_host, pos, S, s_dyn, 0);
+    }
     if (warp < hw) {
-      if (host_dense) host_copy_ordered<kRowsInFlight>(p, n_ord, lane);
+      if (host_dense) host_copy_ordered<kRowsInFlight>(p, n_ord, lane, (uint32_t)(pos * hw + warp));
       else stride_copy(p, bh, n_host, p.base[host_src], (uint32_t)(pos * hw + warp), (uint32_t)(S * hw), lane,
                        p.host_rows);
     } else if (warp < hw + p.n_peers * pw) {
@@ -1358,8 +1452,18 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
   const uint32_t pos = smid < (uint32_t)kMaxSmId ? gp.sm_pos[smid] : blockIdx.x;
   const bool walker = gp.early_walk && pos >= ntiles;
   const uint32_t arrivals = gp.early_walk ? min(gridDim.x, ntiles) : gridDim.x;
+  uint32_t *s_hist = (lp.hist && gp.hist_smem) ? s_dyn : nullptr;  // the range-table area
+  if (s_hist) {
+    for (uint32_t i = threadIdx.x; i < gp.n_ranges; i += blockDim.x) s_hist[i] = 0;
+    __syncthreads();
+  }
   for (uint32_t t = pos; t < ntiles; t += gridDim.x)
-    locate_tile<KeyT, kGatherThreads>(lp, t, s_cnt, s_base);
+    locate_tile<KeyT, kGatherThreads>(lp, t, s_cnt, s_base, s_hist);
+  __syncthreads();
+  if (s_hist && pos < ntiles)
+    for (uint32_t i = threadIdx.x; i < gp.n_ranges; i += blockDim.x)
+      if (s_hist[i]) atomicAdd(&lp.range_count[i], s_hist[i]);
+  if (threadIdx.x == 0) atomicMax(&gp.ctrl->t_loc_max, globaltimer_ns());  // diagnostic stamp
   if (walker) {
     host_walk_copy(gp, threadIdx.x >> 5, threadIdx.x & 31, &gp.ctrl->grid_arrive, arrivals);
     role_wait(&gp.ctrl->grid_arrive, arrivals);
@@ -1451,6 +1555,46 @@ __global__ void __launch_bounds__(32, 1) smid_probe_kernel(uint32_t *smids) {
     uint32_t smid;
     asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
     smids[blockIdx.x] = smid;
+  }
+}
+
+// ---------------------------------------------------------------------------- A0 calibrate
+// Bandwidth vs the number of SMs dedicated to a source (A0, Fig. 6): one CTA per
+// SM (cooperative launch, the gather kernels' shared-memory footprint); the CTA at position
+// pos of the chip-spreading SM order reads for role pos / k (role r < n_roles: source
+// src_id[r]), so each source gets k SMs spread over the chip exactly as the extract
+// kernels place their roles.  A role's warps claim kRowsInFlight entries at a time from its
+// sample list (row << 32 | out row, ascending rows) and copy them with copy_rows.
+struct CalibParams {
+  const uint8_t *base[kMaxSrc];
+  const uint64_t *ents;      // n_roles x n_ents sample entries
+  uint8_t *out;              // n_roles x n_ents rows
+  uint32_t *cursor;          // n_roles claim cursors, zero before the launch
+  uint32_t n_ents;
+  uint32_t row_bytes;
+  int32_t n_roles;
+  int32_t k;                 // SMs per role
+  int32_t src_id[kMaxSrc];
+  uint8_t sm_pos[kMaxSmId];
+};
+
+__global__ void __launch_bounds__(kGatherThreads, 1) calib_kernel(const CalibParams p) {
+  uint32_t smid;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+  const int pos = smid < (uint32_t)kMaxSmId ? p.sm_pos[smid] : (int)blockIdx.x;
+  const int role = pos / p.k;
+  if (role >= p.n_roles) return;
+  const int lane = threadIdx.x & 31;
+  const uint64_t *e = p.ents + (uint64_t)role * p.n_ents;
+  uint8_t *out = p.out + (uint64_t)role * p.n_ents * p.row_bytes;
+  const uint8_t *base = p.base[p.src_id[role]];
+  while (true) {
+    uint32_t e0 = 0;
+    if (lane == 0) e0 = atomicAdd(&p.cursor[role], (uint32_t)kRowsInFlight);
+    e0 = __shfl_sync(kFullMask, e0, 0);
+    if (e0 >= p.n_ents) break;
+    copy_rows<kRowsInFlight>(base, out, p.row_bytes, e + e0, (int)min((uint32_t)kRowsInFlight, p.n_ents - e0),
+                             lane);
   }
 }
 
@@ -1569,15 +1713,33 @@ __global__ void __launch_bounds__(512) msg_copy_kernel(const MsgParams p) {
 }
 
 // ---------------------------------------------------------------------------- refresh
-// Cache refresh, step 1: every key whose location changes is first pointed at
-// the host (which holds every entry), so no reader can reach a slot whose content is about
-// to be rewritten; unchanged locations stay.
+// Cache refresh, hashtable step: every key whose CURRENT location is a GPU slot
+// in [lo, hi) and whose location changes is pointed at the host first (which holds every
+// entry; tier slot tier_slot[k] when the host tier is on, else row = key), so no reader can
+// reach a slot whose content is about to be rewritten.  Unchanged and host keys stay.
 __global__ void __launch_bounds__(256) refresh_evict_kernel(uint64_t *loc, const uint64_t *loc_new,
-                                                            uint64_t N, uint64_t host_tag) {
+                                                            uint64_t N, uint64_t host_tag,
+                                                            const uint32_t *tier_slot, uint64_t G,
+                                                            uint64_t lo, uint64_t hi) {
   for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < N;
        k += (uint64_t)gridDim.x * blockDim.x) {
     const uint64_t a = loc[k];
-    if (a != loc_new[k]) loc[k] = host_tag | k;
+    const uint64_t row = a & UGACHE_LOC_ROW_MASK;
+    if ((a >> UGACHE_LOC_SRC_SHIFT) < G && row >= lo && row < hi && a != loc_new[k])
+      loc[k] = host_tag | (tier_slot ? (uint64_t)tier_slot[k] : k);
+  }
+}
+
+// Cache refresh, install step of a chunk: keys whose NEW location is a GPU slot in [lo, hi)
+// take it (the slot's content was rewritten by its owner before this runs).
+__global__ void __launch_bounds__(256) refresh_install_kernel(uint64_t *loc, const uint64_t *loc_new,
+                                                              uint64_t N, uint64_t G, uint64_t lo,
+                                                              uint64_t hi) {
+  for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < N;
+       k += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t b = loc_new[k];
+    const uint64_t row = b & UGACHE_LOC_ROW_MASK;
+    if ((b >> UGACHE_LOC_SRC_SHIFT) < G && row >= lo && row < hi) loc[k] = b;
   }
 }
 

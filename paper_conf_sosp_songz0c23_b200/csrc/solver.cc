@@ -257,6 +257,10 @@ ugache_status solve(const ugache_config *cfg, int device_sms, const float *hotne
   plan->host_sms = p.host_sms;
   plan->peer_sms = p.peer_sms;
   plan->num_sms = p.S;
+  {
+    const uint64_t be = plan->band_end;
+    plan->host_mass_frac = sw.total > 0 ? std::max(0.0, sw.total - sw.P[be]) / sw.total : 0.0;
+  }
   return UGACHE_OK;
 }
 
@@ -298,13 +302,17 @@ ugache_status build_placement(const ugache_config *cfg, const uint32_t *order,
   return UGACHE_OK;
 }
 
-// tier[t] = table[order[be + t]] for t < N - be (parallel, first touch by the copying thread)
+// tier[t] = table[order[(be + t) mod N]] for t < N (parallel, first touch by the copying
+// thread): the host-resident ranks [be, N) first, in rank order, then the cached ranks
+// [0, be) -- the slots a cache refresh may redirect evicted keys to.
 template <typename OrderT>
 void fill_host_tier_impl(const uint8_t *table, uint32_t R, const OrderT *order, uint64_t be,
                          uint64_t N, uint8_t *tier) {
 #pragma omp parallel for schedule(static)
-  for (int64_t t = 0; t < (int64_t)(N - be); ++t)
-    std::memcpy(tier + (uint64_t)t * R, table + (uint64_t)order[be + (uint64_t)t] * R, R);
+  for (int64_t t = 0; t < (int64_t)N; ++t) {
+    const uint64_t r = ((uint64_t)t + be) % N;
+    std::memcpy(tier + (uint64_t)t * R, table + (uint64_t)order[r] * R, R);
+  }
 }
 
 void fill_host_tier(const uint8_t *table, uint32_t R, const uint64_t *order, uint64_t be,
@@ -349,9 +357,59 @@ ugache_status ugache_build_placement(const ugache_config *cfg, const uint64_t *o
   return ug::build_placement(cfg, ord.data(), plan, gpu, loc, slot_keys, n_slots);
 }
 
+ugache_status ugache_model_time(const ugache_plan *plan, int32_t num_gpus, uint64_t num_rows,
+                                const uint64_t *const *locs, const float *hotness, double *z) {
+  if (!plan || !locs || !z || num_gpus < 1 || num_gpus > UGACHE_MAX_GPUS || num_rows == 0)
+    return UGACHE_EINVAL;
+  const int G = num_gpus, M = G + 1;
+  for (int i = 0; i < G; ++i)
+    if (!locs[i]) return UGACHE_EINVAL;
+  // mass[i][j] = sum of hotness over the keys GPU i reads from source j
+  std::vector<double> mass((size_t)G * M, 0.0);
+  bool ok = true;
+  for (int i = 0; i < G; ++i) {
+    std::vector<double> m(M, 0.0);
+#pragma omp parallel
+    {
+      std::vector<double> part(M, 0.0);
+      bool good = true;
+#pragma omp for schedule(static)
+      for (int64_t k = 0; k < (int64_t)num_rows; ++k) {
+        const uint64_t src = locs[i][k] >> UGACHE_LOC_SRC_SHIFT;
+        const float h = hotness ? hotness[k] : 1.0f;
+        if (src > (uint64_t)G || !std::isfinite(h)) good = false;
+        else part[src] += h > 0.0f ? (double)h : 0.0;
+      }
+#pragma omp critical
+      {
+        for (int j = 0; j < M; ++j) m[j] += part[j];
+        ok = ok && good;
+      }
+    }
+    for (int j = 0; j < M; ++j) mass[(size_t)i * M + j] = m[j];
+  }
+  if (!ok) return UGACHE_EINVAL;
+  // t^j_i = T_{i<-j} * mass, t_i = max(max_j t^j_i, sum_j R_{i<-j} t^j_i), z = max_i t_i
+  double zmax = 0.0;
+  for (int i = 0; i < G; ++i) {
+    double tmax = 0.0, area = 0.0;
+    for (int j = 0; j < M; ++j) {
+      const bool host = j == G, local = j == i;
+      const double T = host ? plan->T_host : (local ? plan->T_local : plan->T_peer);
+      const double Rr = host ? plan->R_host : (local ? plan->R_local : plan->R_peer);
+      const double t = T * mass[(size_t)i * M + j];
+      tmax = std::max(tmax, t);
+      area += Rr * t;
+    }
+    zmax = std::max(zmax, std::max(tmax, area));
+  }
+  *z = zmax;
+  return UGACHE_OK;
+}
+
 uint64_t ugache_host_tier_rows(const ugache_plan *plan, uint64_t num_rows) {
   if (!plan || plan->band_end > num_rows) return 0;
-  return num_rows - plan->band_end;
+  return num_rows;
 }
 
 ugache_status ugache_fill_host_tier(const ugache_config *cfg, const uint64_t *order,
@@ -363,7 +421,6 @@ ugache_status ugache_fill_host_tier(const ugache_config *cfg, const uint64_t *or
   if (st != UGACHE_OK) return st;
   const uint64_t N = cfg->num_rows, be = plan->band_end;
   if (be > N) return UGACHE_EINVAL;
-  if (be == N) return UGACHE_OK;
   if (!tier) return UGACHE_EINVAL;
   ug::fill_host_tier(static_cast<const uint8_t *>(host_table), cfg->row_bytes, order, be, N,
                      static_cast<uint8_t *>(tier));

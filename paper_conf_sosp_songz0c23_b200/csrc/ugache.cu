@@ -29,10 +29,13 @@ struct ugache_ctx {
   const uint8_t *host_table = nullptr;
   const uint8_t *host_table_dev = nullptr;
   std::vector<const void *> pinned;  // host ranges this ctx registered (refcounted globally)
-  // host tier (UGACHE_FLAG_HOST_TIER): rank-ordered copy of the host-resident rows
+  // host tier (UGACHE_FLAG_HOST_TIER): rank-ordered copy of every row, host-resident ranks
+  // first (slot of rank r = (r - band_end) mod N)
   uint8_t *tier_owned = nullptr;
   size_t tier_owned_bytes = 0;
   const uint8_t *tier_dev = nullptr;
+  std::vector<uint32_t> h_tier_slot;  // tier slot of every key (host-side, for refresh)
+  uint32_t *d_tier_slot = nullptr;    // device copy, uploaded by the first refresh
   // this GPU's cache slab and location table
   uint8_t *slab = nullptr;
   uint64_t slab_bytes = 0;
@@ -41,10 +44,12 @@ struct ugache_ctx {
   uint64_t slot_keys_cap = 0;
   std::vector<uint64_t> h_slot_keys;  // host copy of the slot list (refresh diffs)
   uint64_t *d_loc = nullptr;
-  // cache refresh: 0 idle, 1 evicted (LT transitional), 2 content written
+  // cache refresh: 0 idle, 1 evicted (LT transitional), 2 content written,
+  // 3 staged for the chunked protocol (ugache_refresh_chunk)
   int refresh_state = 0;
   uint64_t *d_loc_new = nullptr;
   std::vector<uint64_t> new_slot_keys;
+  std::vector<uint64_t> refresh_slots;  // changed slots of this GPU, ascending
   uint64_t refresh_changed = 0, refresh_pos = 0;
   uint64_t *d_refresh = nullptr;  // changed (slot, key) lists staged for the content step
   // sources
@@ -73,6 +78,9 @@ struct ugache_ctx {
   int wd_host_warps = 1, wd_peer_warps = 1;  // warp-granular dedication: warps per SM
   int host_rows = ugk::kRowsInFlight;        // env UGACHE_HOST_ROWS (1, 2, 4, 8)
   int host_walk = 1;                         // UGACHE_OPT_HOST_WALK
+  int preorder = 1;                          // UGACHE_OPT_PREORDER (env UGACHE_PREORDER)
+  int hist_smem = 1;                         // env UGACHE_HIST_SMEM (fused: per-CTA histogram)
+  int host_segments = 2;                     // env UGACHE_HOST_SEGMENTS (ordered host copy)
   int fused = 2;                             // UGACHE_OPT_FUSED: 0 off, 1 on, 2 auto
   int early_walk = 0;                        // UGACHE_OPT_EARLY_WALK (env UGACHE_EARLY_WALK)
   int local_bulk = 2;                        // UGACHE_OPT_LOCAL_BULK (0 off, 1 on, 2 auto, 3)
@@ -219,7 +227,10 @@ void unpin_all(ugache_ctx *ctx) {
   ctx->pinned.clear();
 }
 
-ugache_status ensure_scratch(ugache_ctx *ctx, uint64_t n) {
+// Scratch of the extract kernels.  The queue sentinels (~0) and sub-queue counters (0) are
+// initialised on the extract stream itself: a caller's non-blocking stream is not ordered
+// after the legacy default stream, so a plain cudaMemset could land after the first launch.
+ugache_status ensure_scratch(ugache_ctx *ctx, uint64_t n, cudaStream_t s) {
   if (n <= ctx->bucket_cap) return UGACHE_OK;
   uint64_t cap = std::max<uint64_t>(n, 1024);
   if (ctx->d_buckets) {
@@ -242,11 +253,11 @@ ugache_status ensure_scratch(ugache_ctx *ctx, uint64_t n) {
   ctx->queue_cap = cap + (uint64_t)(ctx->sm_count + 1) * ugk::kStreamChunk;
   const size_t qbytes = (size_t)(ctx->cfg.num_gpus + 1) * ctx->queue_cap * sizeof(uint64_t);
   UG_CUDA(ctx, cudaMalloc(&ctx->d_queues, qbytes));
-  UG_CUDA(ctx, cudaMemset(ctx->d_queues, 0xFF, qbytes));
+  UG_CUDA(ctx, cudaMemsetAsync(ctx->d_queues, 0xFF, qbytes, s));
   if (!ctx->d_qctr) {
     const size_t cb = 2 * (size_t)ugk::kMaxSrc * ugk::kMaxSmId * sizeof(uint32_t);
     UG_CUDA(ctx, cudaMalloc(&ctx->d_qctr, cb));
-    UG_CUDA(ctx, cudaMemset(ctx->d_qctr, 0, cb));
+    UG_CUDA(ctx, cudaMemsetAsync(ctx->d_qctr, 0, cb, s));
   }
   UG_CUDA(ctx, cudaMalloc(&ctx->d_host_sorted, cap * sizeof(uint64_t)));
   ctx->bucket_cap = cap;
@@ -319,6 +330,18 @@ ugache_status check_given_placement(ugache_ctx *ctx, const ugache_config *cfg, c
   return ok ? UGACHE_OK : fail(ctx, UGACHE_EINVAL, "location table does not resolve every key");
 }
 
+// MemAvailable of /proc/meminfo in bytes (0 if unknown).
+uint64_t host_mem_available() {
+  FILE *f = fopen("/proc/meminfo", "r");
+  if (!f) return 0;
+  char line[256];
+  uint64_t kb = 0;
+  while (fgets(line, sizeof(line), f))
+    if (sscanf(line, "MemAvailable: %lu kB", &kb) == 1) break;
+  fclose(f);
+  return kb * 1024;
+}
+
 ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void *host_table,
                           const std::vector<uint32_t> &order, const void *host_tier,
                           const uint64_t *given_loc = nullptr, const uint64_t *given_slots = nullptr,
@@ -328,10 +351,13 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   ugache_status st = pin_host(ctx, host_table, (size_t)(N * R), &ctx->host_table_dev);
   if (st != UGACHE_OK) return st;
   ctx->host_table = static_cast<const uint8_t *>(host_table);
-  const uint64_t tier_rows = N - ctx->plan.band_end;
-  if ((cfg->flags & UGACHE_FLAG_HOST_TIER) && tier_rows) {
+  const uint64_t tier_rows = N;  // every row (a refresh may send any key to the host)
+  if (cfg->flags & UGACHE_FLAG_HOST_TIER) {
     const void *tier = host_tier;
     if (!tier) {  // build this ctx's own rank-ordered host tier
+      const uint64_t avail = host_mem_available();
+      if (avail && tier_rows * R > avail / 10 * 9)
+        return fail(ctx, UGACHE_ENOMEM, "the host tier (another copy of every row) does not fit host RAM");
       ctx->tier_owned_bytes = (size_t)(tier_rows * R);
       void *m = mmap(nullptr, ctx->tier_owned_bytes, PROT_READ | PROT_WRITE,
                      MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
@@ -347,6 +373,15 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
     }
     st = pin_host(ctx, tier, (size_t)(tier_rows * R), &ctx->tier_dev);
     if (st != UGACHE_OK) return st;
+    try {
+      ctx->h_tier_slot.resize(N);
+    } catch (const std::bad_alloc &) {
+      return fail(ctx, UGACHE_ENOMEM, "host allocation of the tier slot map failed");
+    }
+    const uint64_t be = ctx->plan.band_end;
+#pragma omp parallel for schedule(static)
+    for (int64_t r = 0; r < (int64_t)N; ++r)
+      ctx->h_tier_slot[order[r]] = (uint32_t)(((uint64_t)r + N - be) % N);
   }
 
   // location table and slot list of this rank
@@ -395,9 +430,13 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   UG_CUDA(ctx, cudaMalloc(&ctx->d_ranges, 2 * ugk::kMaxRanges * sizeof(uint32_t)));
   UG_CUDA(ctx, cudaMemset(ctx->d_ranges, 0, 2 * ugk::kMaxRanges * sizeof(uint32_t)));
   // host key ranges: the smallest power-of-two rows per range giving <= kMaxRanges ranges
-  ctx->range_shift = 0;
-  while (((N - 1) >> ctx->range_shift) + 1 > (uint64_t)ugk::kMaxRanges) ++ctx->range_shift;
-  ctx->n_ranges = (uint32_t)(((N - 1) >> ctx->range_shift) + 1);
+  // over the host source's rows (the tier's slots when it is on, else the table's keys)
+  {
+    const uint64_t hr = std::max<uint64_t>(N, 1);
+    ctx->range_shift = 0;
+    while (((hr - 1) >> ctx->range_shift) + 1 > (uint64_t)ugk::kMaxRanges) ++ctx->range_shift;
+    ctx->n_ranges = (uint32_t)(((hr - 1) >> ctx->range_shift) + 1);
+  }
   {  // ordering pays once host rows share translation pages: >= 1 key per 2 MB of host source
     const uint64_t host_rows = ctx->tier_dev ? N - ctx->plan.band_end : N;
     const uint64_t pages = (host_rows * R) >> 21;
@@ -408,6 +447,9 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_HOST_DYNAMIC")) ctx->host_dynamic = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_HOST_ROWS")) ctx->host_rows = atoi(e);
   if (const char *e = getenv("UGACHE_EARLY_WALK")) ctx->early_walk = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_PREORDER")) ctx->preorder = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_HIST_SMEM")) ctx->hist_smem = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_HOST_SEGMENTS")) ctx->host_segments = std::max(1, std::min(8, atoi(e)));
   if (const char *e = getenv("UGACHE_LOCAL_BULK")) ctx->local_bulk = std::max(0, std::min(3, atoi(e)));
   if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_STREAM_K")) ctx->stream_k = std::max(1, std::min(ugk::kStreamK, atoi(e)));
@@ -507,6 +549,9 @@ static ugache_status init_impl(ugache_ctx **out, const ugache_config *cfg, const
                                const uint64_t *given_slots = nullptr, uint64_t given_n = 0) {
   if (!out || !cfg || !host_table) return UGACHE_EINVAL;
   *out = nullptr;
+  // rows are read with 16-byte vector loads and cp.async.bulk: 16-byte aligned sources only
+  if (reinterpret_cast<uintptr_t>(host_table) % 16 || reinterpret_cast<uintptr_t>(host_tier) % 16)
+    return UGACHE_EINVAL;
   if (cfg->rank < 0 || cfg->rank >= cfg->num_gpus) return UGACHE_EINVAL;
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= 0) {
@@ -544,14 +589,22 @@ static ugache_status init_impl(ugache_ctx **out, const ugache_config *cfg, const
       ug::Params p;
       st = ug::resolve_params(cfg, ctx->sm_count, &p);
       if (st == UGACHE_OK) {
+        // order must be a permutation of [0, N): a key missing from it would keep a host
+        // location whose tier slot lies outside the tier
         order.resize(cfg->num_rows);
+        std::vector<uint8_t> seen(cfg->num_rows, 0);
         for (uint64_t i = 0; i < cfg->num_rows; ++i) {
-          if (order_in[i] >= cfg->num_rows) { st = UGACHE_EINVAL; break; }
+          if (order_in[i] >= cfg->num_rows || seen[order_in[i]]) { st = UGACHE_EINVAL; break; }
+          seen[order_in[i]] = 1;
           order[i] = (uint32_t)order_in[i];
         }
         ctx->plan = *plan_in;
         if (plan_in->num_gpus != cfg->num_gpus || plan_in->host_sms != p.host_sms ||
             plan_in->peer_sms != p.peer_sms)
+          st = UGACHE_EINVAL;
+        const uint64_t cap = std::min<uint64_t>(cfg->capacity_rows, cfg->num_rows);
+        if (plan_in->capacity_rows > cap || plan_in->k > plan_in->capacity_rows ||
+            plan_in->band_end < plan_in->k || plan_in->band_end > cfg->num_rows)
           st = UGACHE_EINVAL;
         if (plan_in->num_sms > ctx->sm_count) st = UGACHE_EINVAL;
       }
@@ -642,7 +695,7 @@ ugache_status ugache_set_peer_slabs(ugache_ctx *ctx, const void *const *slabs) {
   if (!ctx || !slabs) return UGACHE_EINVAL;
   for (int j = 0; j < ctx->cfg.num_gpus; ++j) {
     if (j == ctx->cfg.rank) continue;
-    if (!slabs[j]) return UGACHE_EINVAL;
+    if (!slabs[j] || reinterpret_cast<uintptr_t>(slabs[j]) % 16) return UGACHE_EINVAL;
     int dev = -1;
     if (!is_device_pointer(slabs[j], &dev)) return fail(ctx, UGACHE_EPEER, "peer slab is not device memory");
     if (dev != ctx->device) {
@@ -686,26 +739,99 @@ ugache_status ugache_fill(ugache_ctx *ctx, void *stream) {
 }
 
 // ---- cache refresh (section 7.2) -------------------------------------------
-ugache_status ugache_refresh_begin(ugache_ctx *ctx, const uint64_t *new_loc,
-                                   const uint64_t *new_slot_keys, uint64_t n_new_slots,
-                                   void *stream) {
-  if (!ctx || !new_loc) return UGACHE_EINVAL;
+namespace {
+// Host location of key k while a refresh redirects it: the tier slot, or the key itself.
+uint64_t host_entry(const ugache_ctx *ctx, uint64_t k) {
+  const uint64_t tag = (uint64_t)ctx->cfg.num_gpus << UGACHE_LOC_SRC_SHIFT;
+  return tag | (ctx->tier_dev ? (uint64_t)ctx->h_tier_slot[k] : k);
+}
+
+// Stage a new placement: checked like ugache_init_with_placement (host rows = keys), its
+// host rows translated to tier slots when the ctx has a tier, uploaded next to the current
+// table; the changed slots of this GPU (slot, new key) uploaded for the content steps.
+ugache_status refresh_stage(ugache_ctx *ctx, const uint64_t *new_loc, const uint64_t *new_slot_keys,
+                            uint64_t n_new_slots, cudaStream_t s) {
   if (ctx->refresh_state != 0) return fail(ctx, UGACHE_ESTATE, "refresh already in progress");
   if (!ctx->filled) return fail(ctx, UGACHE_ESTATE, "refresh before fill");
-  if (ctx->tier_dev) return fail(ctx, UGACHE_EINVAL, "refresh of a host-tier ctx is not supported");
   ugache_status st = check_given_placement(ctx, &ctx->cfg, new_loc, new_slot_keys, n_new_slots);
   if (st != UGACHE_OK) return st;
   st = begin(ctx);
   if (st != UGACHE_OK) return st;
   const uint64_t N = ctx->cfg.num_rows;
-  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const int G = ctx->cfg.num_gpus;
   UG_CUDA(ctx, cudaStreamSynchronize(s));
   if (!ctx->d_loc_new) UG_CUDA(ctx, cudaMalloc(&ctx->d_loc_new, N * sizeof(uint64_t)));
-  UG_CUDA(ctx, cudaMemcpy(ctx->d_loc_new, new_loc, N * sizeof(uint64_t), cudaMemcpyHostToDevice));
+  if (ctx->tier_dev) {
+    std::vector<uint64_t> tr(N);
+#pragma omp parallel for schedule(static)
+    for (int64_t k = 0; k < (int64_t)N; ++k)
+      tr[k] = (new_loc[k] >> UGACHE_LOC_SRC_SHIFT) == (uint64_t)G ? host_entry(ctx, (uint64_t)k) : new_loc[k];
+    UG_CUDA(ctx, cudaMemcpy(ctx->d_loc_new, tr.data(), N * sizeof(uint64_t), cudaMemcpyHostToDevice));
+    if (!ctx->d_tier_slot) {
+      UG_CUDA(ctx, cudaMalloc(&ctx->d_tier_slot, N * sizeof(uint32_t)));
+      UG_CUDA(ctx, cudaMemcpy(ctx->d_tier_slot, ctx->h_tier_slot.data(), N * sizeof(uint32_t),
+                              cudaMemcpyHostToDevice));
+    }
+  } else {
+    UG_CUDA(ctx, cudaMemcpy(ctx->d_loc_new, new_loc, N * sizeof(uint64_t), cudaMemcpyHostToDevice));
+  }
   ctx->new_slot_keys.assign(new_slot_keys, new_slot_keys + n_new_slots);
-  const uint64_t host_tag = (uint64_t)ctx->cfg.num_gpus << UGACHE_LOC_SRC_SHIFT;
-  ugk::refresh_evict_kernel<<<ctx->sm_count * 8, 256, 0, s>>>(ctx->d_loc, ctx->d_loc_new, N, host_tag);
+  std::vector<uint64_t> keys;
+  ctx->refresh_slots.clear();
+  for (uint64_t i = 0; i < ctx->new_slot_keys.size(); ++i)
+    if (i >= ctx->h_slot_keys.size() || ctx->h_slot_keys[i] != ctx->new_slot_keys[i]) {
+      ctx->refresh_slots.push_back(i);
+      keys.push_back(ctx->new_slot_keys[i]);
+    }
+  ctx->refresh_changed = ctx->refresh_slots.size();
+  ctx->refresh_pos = 0;
+  cudaFree(ctx->d_refresh);
+  ctx->d_refresh = nullptr;
+  UG_CUDA(ctx, cudaMalloc(&ctx->d_refresh, 2 * std::max<size_t>(keys.size(), 1) * sizeof(uint64_t)));
+  if (!keys.empty()) {
+    UG_CUDA(ctx, cudaMemcpy(ctx->d_refresh, ctx->refresh_slots.data(), keys.size() * 8, cudaMemcpyHostToDevice));
+    UG_CUDA(ctx, cudaMemcpy(ctx->d_refresh + keys.size(), keys.data(), keys.size() * 8, cudaMemcpyHostToDevice));
+  }
+  return UGACHE_OK;
+}
+
+// Keys whose current location is a GPU slot in [lo, hi) and changes -> host (the host holds
+// every entry), so nobody reaches those slots while their content is rewritten.
+ugache_status refresh_evict(ugache_ctx *ctx, uint64_t lo, uint64_t hi, cudaStream_t s) {
+  ugk::refresh_evict_kernel<<<ctx->sm_count * 8, 256, 0, s>>>(
+      ctx->d_loc, ctx->d_loc_new, ctx->cfg.num_rows, (uint64_t)ctx->cfg.num_gpus << UGACHE_LOC_SRC_SHIFT,
+      ctx->tier_dev ? ctx->d_tier_slot : nullptr, (uint64_t)ctx->cfg.num_gpus, lo, hi);
   UG_CUDA(ctx, cudaGetLastError());
+  return UGACHE_OK;
+}
+
+// Rewrite the changed slots of this GPU with index in [a, b) of the changed list.
+ugache_status refresh_fill(ugache_ctx *ctx, uint64_t a, uint64_t b, int32_t max_sms, cudaStream_t s) {
+  if (b <= a) return UGACHE_OK;
+  ugk::FillParams fp;
+  fp.slot_idx = ctx->d_refresh + a;
+  fp.slot_keys = ctx->d_refresh + ctx->refresh_changed + a;
+  fp.table = ctx->host_table_dev;
+  fp.slab = ctx->slab;
+  fp.n_slots = b - a;
+  fp.row_bytes = ctx->cfg.row_bytes;
+  // throttle: at most max_sms SMs' worth of CTAs
+  const int sms = max_sms ? std::min<int>(max_sms, ctx->sm_count) : ctx->sm_count;
+  ugk::fill_kernel<<<sms * 8, 256, 0, s>>>(fp);
+  UG_CUDA(ctx, cudaGetLastError());
+  return UGACHE_OK;
+}
+}  // namespace
+
+ugache_status ugache_refresh_begin(ugache_ctx *ctx, const uint64_t *new_loc,
+                                   const uint64_t *new_slot_keys, uint64_t n_new_slots,
+                                   void *stream) {
+  if (!ctx || !new_loc) return UGACHE_EINVAL;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  ugache_status st = refresh_stage(ctx, new_loc, new_slot_keys, n_new_slots, s);
+  if (st != UGACHE_OK) return st;
+  st = refresh_evict(ctx, 0, ~0ull, s);
+  if (st != UGACHE_OK) return st;
   ctx->refresh_state = 1;
   return UGACHE_OK;
 }
@@ -716,53 +842,54 @@ ugache_status ugache_refresh_content(ugache_ctx *ctx, int32_t max_sms, uint64_t 
   if (ctx->refresh_state != 1) return fail(ctx, UGACHE_ESTATE, "refresh_content before refresh_begin");
   ugache_status st = begin(ctx);
   if (st != UGACHE_OK) return st;
-  cudaStream_t s = static_cast<cudaStream_t>(stream);
-  if (!ctx->d_refresh) {  // first call: the changed slots, staged on the device once
-    std::vector<uint64_t> idx, keys;
-    for (uint64_t i = 0; i < ctx->new_slot_keys.size(); ++i)
-      if (i >= ctx->h_slot_keys.size() || ctx->h_slot_keys[i] != ctx->new_slot_keys[i]) {
-        idx.push_back(i);
-        keys.push_back(ctx->new_slot_keys[i]);
-      }
-    ctx->refresh_changed = idx.size();
-    ctx->refresh_pos = 0;
-    UG_CUDA(ctx, cudaMalloc(&ctx->d_refresh, 2 * std::max<size_t>(idx.size(), 1) * sizeof(uint64_t)));
-    if (!idx.empty()) {
-      UG_CUDA(ctx, cudaMemcpy(ctx->d_refresh, idx.data(), idx.size() * 8, cudaMemcpyHostToDevice));
-      UG_CUDA(ctx, cudaMemcpy(ctx->d_refresh + idx.size(), keys.data(), keys.size() * 8,
-                              cudaMemcpyHostToDevice));
-    }
-  }
-  const uint64_t total = ctx->refresh_changed;
-  const uint64_t lo = ctx->refresh_pos;
+  const uint64_t total = ctx->refresh_changed, lo = ctx->refresh_pos;
   const uint64_t hi = max_rows ? std::min(total, lo + max_rows) : total;
-  if (hi > lo) {
-    ugk::FillParams fp;
-    fp.slot_idx = ctx->d_refresh + lo;
-    fp.slot_keys = ctx->d_refresh + total + lo;
-    fp.table = ctx->host_table_dev;
-    fp.slab = ctx->slab;
-    fp.n_slots = hi - lo;
-    fp.row_bytes = ctx->cfg.row_bytes;
-    // throttle: at most max_sms SMs' worth of CTAs, max_rows rows per call
-    const int sms = max_sms ? std::min(max_sms, ctx->sm_count) : ctx->sm_count;
-    ugk::fill_kernel<<<sms * 8, 256, 0, s>>>(fp);
-    UG_CUDA(ctx, cudaGetLastError());
-    UG_CUDA(ctx, cudaStreamSynchronize(s));
-  }
+  st = refresh_fill(ctx, lo, hi, max_sms, static_cast<cudaStream_t>(stream));  // asynchronous
+  if (st != UGACHE_OK) return st;
   ctx->refresh_pos = hi;
   if (remaining) *remaining = total - hi;
-  if (hi == total) {
-    cudaFree(ctx->d_refresh);
-    ctx->d_refresh = nullptr;
-    ctx->refresh_state = 2;
-  }
+  if (hi == total) ctx->refresh_state = 2;
   return UGACHE_OK;
+}
+
+ugache_status ugache_refresh_stage(ugache_ctx *ctx, const uint64_t *new_loc,
+                                   const uint64_t *new_slot_keys, uint64_t n_new_slots,
+                                   void *stream) {
+  if (!ctx || !new_loc) return UGACHE_EINVAL;
+  ugache_status st = refresh_stage(ctx, new_loc, new_slot_keys, n_new_slots, static_cast<cudaStream_t>(stream));
+  if (st != UGACHE_OK) return st;
+  ctx->refresh_state = 3;
+  return UGACHE_OK;
+}
+
+ugache_status ugache_refresh_chunk(ugache_ctx *ctx, int32_t step, uint64_t slot_lo, uint64_t slot_hi,
+                                   int32_t max_sms, void *stream) {
+  if (!ctx || max_sms < 0 || slot_hi < slot_lo) return UGACHE_EINVAL;
+  if (ctx->refresh_state != 3) return fail(ctx, UGACHE_ESTATE, "refresh_chunk before refresh_stage");
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  switch (step) {
+    case UGACHE_REFRESH_EVICT: return refresh_evict(ctx, slot_lo, slot_hi, s);
+    case UGACHE_REFRESH_FILL: {
+      const auto &v = ctx->refresh_slots;
+      const uint64_t a = (uint64_t)(std::lower_bound(v.begin(), v.end(), slot_lo) - v.begin());
+      const uint64_t b = (uint64_t)(std::lower_bound(v.begin(), v.end(), slot_hi) - v.begin());
+      return refresh_fill(ctx, a, b, max_sms, s);
+    }
+    case UGACHE_REFRESH_INSTALL:
+      ugk::refresh_install_kernel<<<ctx->sm_count * 8, 256, 0, s>>>(
+          ctx->d_loc, ctx->d_loc_new, ctx->cfg.num_rows, (uint64_t)ctx->cfg.num_gpus, slot_lo, slot_hi);
+      UG_CUDA(ctx, cudaGetLastError());
+      return UGACHE_OK;
+  }
+  return UGACHE_EINVAL;
 }
 
 ugache_status ugache_refresh_commit(ugache_ctx *ctx, void *stream) {
   if (!ctx) return UGACHE_EINVAL;
-  if (ctx->refresh_state != 2) return fail(ctx, UGACHE_ESTATE, "refresh_commit before refresh_content");
+  if (ctx->refresh_state != 2 && ctx->refresh_state != 3)
+    return fail(ctx, UGACHE_ESTATE, "refresh_commit before refresh_content / refresh_stage");
   ugache_status st = begin(ctx);
   if (st != UGACHE_OK) return st;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
@@ -782,11 +909,172 @@ ugache_status ugache_refresh_commit(ugache_ctx *ctx, void *stream) {
   UG_CUDA(ctx, cudaStreamSynchronize(s));
   ctx->h_slot_keys.swap(ctx->new_slot_keys);
   ctx->new_slot_keys.clear();
+  ctx->refresh_slots.clear();
   ctx->n_slots = ns;
   cudaFree(ctx->d_loc_new);
   ctx->d_loc_new = nullptr;
+  cudaFree(ctx->d_refresh);
+  ctx->d_refresh = nullptr;
   ctx->plan.policy = -1;  // the placement no longer comes from this ctx's solve
   ctx->refresh_state = 0;
+  return UGACHE_OK;
+}
+
+// ---- A0 calibration (Fig. 6) ------------------------------------------------
+namespace {
+uint64_t calib_mix(uint64_t &x) {  // splitmix64 step (sample rows only)
+  uint64_t z = (x += 0x9E3779B97F4A7C15ull);
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+// n sorted uniform random rows of [0, span) as sample entries (row << 32 | i)
+void calib_sample(std::vector<uint64_t> &ents, uint64_t span, uint32_t n, uint64_t seed) {
+  std::vector<uint64_t> rows(n);
+  for (uint32_t i = 0; i < n; ++i) rows[i] = span ? calib_mix(seed) % span : 0;
+  std::sort(rows.begin(), rows.end());
+  const size_t off = ents.size();
+  ents.resize(off + n);
+  for (uint32_t i = 0; i < n; ++i) ents[off + i] = (rows[i] << 32) | i;
+}
+
+// The swept point whose bandwidth first reaches 90 % of the best one (reading R13).
+int calib_pick(const int32_t *ks, const double *bw, int n) {
+  double best = 0;
+  for (int i = 0; i < n; ++i) best = std::max(best, bw[i]);
+  for (int i = 0; i < n; ++i)
+    if (bw[i] >= 0.9 * best) return i;
+  return n - 1;
+}
+}  // namespace
+
+ugache_status ugache_calibrate(ugache_ctx *ctx, uint32_t sample_rows, ugache_calibration *out) {
+  if (!ctx || !out) return UGACHE_EINVAL;
+  if (!ctx->filled || !ctx->peers_ready) return fail(ctx, UGACHE_ESTATE, "calibrate before fill/peers");
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  std::memset(out, 0, sizeof(*out));
+  const uint32_t n = sample_rows ? std::min<uint32_t>(sample_rows, 1u << 22) : 65536u;
+  const int G = ctx->cfg.num_gpus, me = ctx->cfg.rank;
+  const uint32_t R = ctx->cfg.row_bytes;
+  const uint64_t N = ctx->cfg.num_rows;
+  const int roles_max = std::max(1, G - 1);
+  ugk::CalibParams cp{};
+  int S = 0;
+  {
+    ugk::GatherParams gp{};
+    build_roles(ctx, &gp, &S);
+    std::memcpy(cp.sm_pos, gp.sm_pos, sizeof(cp.sm_pos));
+  }
+  for (int j = 0; j < ugk::kMaxSrc; ++j) cp.base[j] = ctx->src_base[j];
+  cp.n_ents = n;
+  cp.row_bytes = R;
+  uint64_t *d_ents = nullptr;
+  uint8_t *d_out = nullptr, *d_flush = nullptr;
+  uint32_t *d_cursor = nullptr;
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  const size_t flush_bytes = 256u << 20;
+  auto cleanup = [&]() {
+    cudaFree(d_ents);
+    cudaFree(d_out);
+    cudaFree(d_flush);
+    cudaFree(d_cursor);
+    if (e0) cudaEventDestroy(e0);
+    if (e1) cudaEventDestroy(e1);
+  };
+  cudaError_t ce = cudaMalloc(&d_ents, (size_t)roles_max * n * sizeof(uint64_t));
+  if (ce == cudaSuccess) ce = cudaMalloc(&d_out, (size_t)roles_max * n * R);
+  if (ce == cudaSuccess) ce = cudaMalloc(&d_flush, flush_bytes);
+  if (ce == cudaSuccess) ce = cudaMalloc(&d_cursor, ugk::kMaxSrc * sizeof(uint32_t));
+  if (ce == cudaSuccess) ce = cudaEventCreate(&e0);
+  if (ce == cudaSuccess) ce = cudaEventCreate(&e1);
+  if (ce == cudaSuccess)
+    ce = cudaFuncSetAttribute(ugk::calib_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOneCtaPerSmSmem);
+  if (ce != cudaSuccess) {
+    cleanup();
+    return cuda_fail(ctx, ce, "calibration buffers");
+  }
+  cp.ents = d_ents;
+  cp.out = d_out;
+  cp.cursor = d_cursor;
+  // time one configuration: median of 3 cold launches (L2 flushed before each), bytes/s
+  auto run = [&](int k, int n_roles, double *bw) -> cudaError_t {
+    cp.k = k;
+    cp.n_roles = n_roles;
+    float ms[3];
+    for (int rep = 0; rep < 3; ++rep) {
+      cudaError_t e = cudaMemsetAsync(d_flush, rep + 1, flush_bytes, nullptr);
+      if (e == cudaSuccess) e = cudaMemsetAsync(d_cursor, 0, ugk::kMaxSrc * sizeof(uint32_t), nullptr);
+      if (e == cudaSuccess) e = cudaEventRecord(e0, nullptr);
+      void *args[] = {&cp};
+      if (e == cudaSuccess)
+        e = cudaLaunchCooperativeKernel((const void *)ugk::calib_kernel, dim3(S), dim3(ugk::kGatherThreads), args,
+                                        kOneCtaPerSmSmem, nullptr);
+      if (e == cudaSuccess) e = cudaEventRecord(e1, nullptr);
+      if (e == cudaSuccess) e = cudaEventSynchronize(e1);
+      if (e == cudaSuccess) e = cudaEventElapsedTime(&ms[rep], e0, e1);
+      if (e != cudaSuccess) return e;
+    }
+    std::sort(ms, ms + 3);
+    *bw = (double)n_roles * n * R / (ms[1] * 1e-3);
+    return cudaSuccess;
+  };
+  std::vector<uint64_t> ents;
+  uint64_t seed = 0x55474143ull ^ ((uint64_t)me << 32);
+  // host source: uniform rows of the whole host source, sorted (range-ordered reads)
+  calib_sample(ents, N, n, seed++);
+  ce = cudaMemcpy(d_ents, ents.data(), ents.size() * 8, cudaMemcpyHostToDevice);
+  cp.src_id[0] = G;
+  const int host_ks[] = {1, 2, 3, 4, 6, 8, 10, 12, 14, 16, 20, 24, 32, 48, 64, 96, 128, 148};
+  for (int k : host_ks) {
+    if (ce != cudaSuccess || k > S || out->n_host_points >= UGACHE_CALIB_MAX_POINTS) break;
+    double bw = 0;
+    ce = run(k, 1, &bw);
+    out->host_points_sms[out->n_host_points] = k;
+    out->host_points_bw[out->n_host_points++] = bw;
+  }
+  if (ce == cudaSuccess && out->n_host_points) {
+    const int i = calib_pick(out->host_points_sms, out->host_points_bw, out->n_host_points);
+    out->host_sms = out->host_points_sms[i];
+    out->bw_host = out->host_points_bw[i];
+  }
+  // local slab: every SM
+  if (ce == cudaSuccess) {
+    ents.clear();
+    calib_sample(ents, std::max<uint64_t>(ctx->n_slots, 1), n, seed++);
+    ce = cudaMemcpy(d_ents, ents.data(), ents.size() * 8, cudaMemcpyHostToDevice);
+    cp.src_id[0] = me;
+    if (ce == cudaSuccess) ce = run(S, 1, &out->bw_local);
+  }
+  // peers: all at once, k SMs per peer (all-to-all ingress)
+  if (ce == cudaSuccess && G > 1) {
+    ents.clear();
+    int r = 0;
+    for (int j = 0; j < G; ++j) {
+      if (j == me) continue;
+      calib_sample(ents, std::max<uint64_t>(ctx->plan.capacity_rows, 1), n, seed++);
+      cp.src_id[r++] = j;
+    }
+    ce = cudaMemcpy(d_ents, ents.data(), ents.size() * 8, cudaMemcpyHostToDevice);
+    const int kmax = std::max(1, (S - std::max(out->host_sms, 1)) / (G - 1));
+    const int peer_ks[] = {1, 2, 3, 4, 6, 8, 10, 12, 16, 20, 24, 32, 40, 48, 64, 96, 128, 148};
+    for (int k : peer_ks) {
+      if (ce != cudaSuccess || k > kmax || out->n_peer_points >= UGACHE_CALIB_MAX_POINTS) break;
+      double bw = 0;
+      ce = run(k, G - 1, &bw);
+      out->peer_points_sms[out->n_peer_points] = k;
+      out->peer_points_bw[out->n_peer_points++] = bw;
+    }
+    if (ce == cudaSuccess && out->n_peer_points) {
+      const int i = calib_pick(out->peer_points_sms, out->peer_points_bw, out->n_peer_points);
+      out->peer_sms = out->peer_points_sms[i];
+      out->bw_peer = out->peer_points_bw[i];
+    }
+  }
+  out->sample_rows = n;
+  cleanup();
+  if (ce != cudaSuccess) return cuda_fail(ctx, ce, "calibration");
   return UGACHE_OK;
 }
 
@@ -819,6 +1107,7 @@ ugache_status ugache_set_option(ugache_ctx *ctx, int32_t option, int64_t value) 
       ctx->host_warps = (int)value;
       return UGACHE_OK;
     case UGACHE_OPT_HOST_WALK: ctx->host_walk = value != 0; return UGACHE_OK;
+    case UGACHE_OPT_PREORDER: ctx->preorder = value != 0; return UGACHE_OK;
     case UGACHE_OPT_FUSED:
       if (value < 0 || value > 2) return UGACHE_EINVAL;
       ctx->fused = (int)value;
@@ -869,6 +1158,8 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
   ctx->timing_valid = false;
   if (n == 0) return UGACHE_OK;
   if (!keys || !out) return UGACHE_EINVAL;
+  if (reinterpret_cast<uintptr_t>(keys) % (key_type == UGACHE_KEY_I64 ? 8 : 4))
+    return fail(ctx, UGACHE_EINVAL, "keys must be aligned to the key size");
   ugache_status st = begin(ctx);
   if (st != UGACHE_OK) return st;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
@@ -923,7 +1214,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     UG_CUDA(ctx, cudaGetLastError());
     ctx->last_launches = 1;
   } else {
-    st = ensure_scratch(ctx, n);
+    st = ensure_scratch(ctx, n, s);
     if (st != UGACHE_OK) return st;
     ugk::LocateParams lp;
     lp.keys = dkeys;
@@ -936,6 +1227,9 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     lp.n = (uint32_t)n;
     lp.row_bytes = R;
     lp.num_src = ctx->cfg.num_gpus + 1;
+    lp.hist = 0;
+    lp.range_shift = ctx->range_shift;
+    lp.range_count = ctx->d_ranges;
     ugk::GatherParams gp;
     gp.buckets = ctx->d_buckets;
     gp.ctrl = ctx->d_ctrl;
@@ -988,6 +1282,9 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     gp.stream_nap = ctx->stream_nap;
     gp.stream_prefetch = ctx->stream_prefetch;
     gp.stream_queues = (!gp.inline_host && ctx->host_sms > 0) || (!gp.inline_peer && ctx->cfg.num_gpus > 1);
+    gp.preorder = 0;
+    gp.hist_smem = ctx->hist_smem;
+    gp.host_segments = ctx->host_segments;
     int grid = 0;
     build_roles(ctx, &gp, &grid);
     if (msg_local) {  // message baseline: no SM reads a peer; the peer buckets stay for msg_*
@@ -1000,15 +1297,26 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     // above 1 KB stay on the two-phase path (measured faster there)
     bool stream = !msg_local && !ctx->warp_dedication && ctx->stream != 0;
     if (stream && ctx->stream == 2) {
+      // Expected host keys of this batch: scaled from the previous launch on this ctx (its
+      // counts mirrored to pinned host memory by the kernel, no synchronisation), or, before
+      // the first launch, from the plan's host hotness mass (keys x host_mass_frac).
       const volatile uint32_t *m = ctx->h_mirror;
       const uint64_t pn = m[0], ph = m[1];
+      const double exp_host = (m[2] && pn) ? (double)ph * (double)n / (double)pn
+                                           : (double)n * ctx->plan.host_mass_frac;
       // with peer rows queued to dedicated SMs the two-phase kernel measured faster (fake
       // peers), so auto takes the single pass only without peer queues
       const bool peer_queues = ctx->cfg.num_gpus > 1 && !(ctx->inline_mask & UGACHE_INLINE_PEERS);
       stream = R <= kStreamAutoMaxRow && !peer_queues &&
-               !(m[2] && pn && ctx->host_sort && ph * n >= (uint64_t)ctx->host_sort_min * pn);
+               !(ctx->host_sort && exp_host >= (double)ctx->host_sort_min);
     }
     const bool fused = ctx->fused == 1 || (ctx->fused == 2 && n <= kFusedAutoMaxKeys);
+    if (!stream && ctx->preorder && ctx->host_sort && !gp.early_walk) {
+      // two-phase paths: the locate pass builds the host range histogram, and every CTA of the
+      // gather scatters a slice of the host bucket into range order (kernels.cuh preorder_host)
+      lp.hist = 1;
+      gp.preorder = 1;
+    }
     if (stream) {  // K3: one cooperative launch, no grid barrier
       if (ctx->timing) {
         UG_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
@@ -1240,6 +1548,8 @@ ugache_status ugache_last_batch_phases(ugache_ctx *ctx, float *ms) {
   ms[0] = rel(c.t_located);
   ms[1] = rel(c.t_ordered);
   ms[2] = rel(c.t_host_done);
+  ms[3] = rel(c.t_loc_last);
+  ms[4] = rel(c.t_end);
   return UGACHE_OK;
 }
 
@@ -1305,6 +1615,7 @@ ugache_status ugache_destroy(ugache_ctx *ctx) {
     cudaFree(ctx->d_ranges);
     cudaFree(ctx->d_loc_new);
     cudaFree(ctx->d_refresh);
+    cudaFree(ctx->d_tier_slot);
     for (int i = 0; i < 3; ++i)
       if (ctx->ev[i]) cudaEventDestroy(ctx->ev[i]);
   }

@@ -74,6 +74,24 @@ def sum_over_ranks(value: float) -> float:
     return _reduce(value, "SUM")
 
 
+def gather_rows(values) -> np.ndarray:
+    """All ranks' copies of a per-rank 1-D float vector, as a [world, len] float64 array
+    (a SUM all-reduce of a matrix whose row r only rank r fills; gloo or NCCL)."""
+    import torch
+    import torch.distributed as dist
+    v = np.asarray(values, dtype=np.float64).ravel()
+    rank, ws = world()
+    if ws == 1:
+        return v[None, :].copy()
+    dev = "cpu"
+    if dist.get_backend() == "nccl":
+        dev = torch.device("cuda", torch.cuda.current_device())
+    m = torch.zeros((ws, len(v)), dtype=torch.float64, device=dev)
+    m[rank] = torch.from_numpy(v).to(dev)
+    dist.all_reduce(m, op=dist.ReduceOp.SUM)
+    return m.cpu().numpy()
+
+
 def connect(cache, group=None, order: Optional[np.ndarray] = None):
     """Exchange slab IPC handles and map every peer (ugache_open_peers)."""
     _, ws = world()

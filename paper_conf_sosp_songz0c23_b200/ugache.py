@@ -53,12 +53,24 @@ def make_config(num_rows: int, row_bytes: int, capacity_rows: int, num_gpus: int
                          flags=_abi.FLAG_HOST_TIER if host_tier else 0)
 
 
+def model_time(plan: ugache_plan, locs, hotness: Optional[np.ndarray]) -> float:
+    """Section 6.2 model value z of a placement (one location table per GPU) under hotness,
+    with plan's T / R (ugache_model_time)."""
+    arrs = [np.ascontiguousarray(l, dtype=np.uint64) for l in locs]
+    ptrs = (ctypes.c_void_p * len(arrs))(*[a.ctypes.data for a in arrs])
+    h = None if hotness is None else np.ascontiguousarray(hotness, dtype=np.float32)
+    z = ctypes.c_double()
+    check(lib().ugache_model_time(ctypes.byref(plan), len(arrs), len(arrs[0]), ctypes.cast(ptrs, ctypes.c_void_p),
+                                  _ptr(h), ctypes.byref(z)), "ugache_model_time")
+    return float(z.value)
+
+
 def host_tier_rows(plan: ugache_plan, num_rows: int) -> int:
     return int(lib().ugache_host_tier_rows(ctypes.byref(plan), num_rows))
 
 
 def fill_host_tier(cfg: ugache_config, order: np.ndarray, plan: ugache_plan, table, tier):
-    """Host-only: tier[t] = table[order[band_end + t]] (ugache_fill_host_tier)."""
+    """Host-only: tier[t] = table[order[(band_end + t) mod N]] for t < N (ugache_fill_host_tier)."""
     order = np.ascontiguousarray(order, dtype=np.uint64)
     check(lib().ugache_fill_host_tier(ctypes.byref(cfg), _ptr(order), ctypes.byref(plan),
                                       _ptr(table), _ptr(tier)), "ugache_fill_host_tier")
@@ -166,9 +178,33 @@ class UGache:
                                            _stream_handle(stream)), "ugache_refresh_content", self.ctx)
         return int(rem.value)
 
+    def refresh_stage(self, loc: np.ndarray, slot_keys: np.ndarray, stream=None):
+        """Chunked refresh: stage the new placement (ugache_refresh_stage)."""
+        loc = np.ascontiguousarray(loc, dtype=np.uint64)
+        sk = np.ascontiguousarray(slot_keys, dtype=np.uint64)
+        check(lib().ugache_refresh_stage(self.ctx, _ptr(loc), _ptr(sk), len(sk), _stream_handle(stream)),
+              "ugache_refresh_stage", self.ctx)
+
+    def refresh_chunk(self, step: str, lo: int, hi: int, max_sms: int = 0, stream=None):
+        """One step ('evict', 'fill', 'install') of the chunked refresh on slots [lo, hi)."""
+        st = {"evict": _abi.REFRESH_EVICT, "fill": _abi.REFRESH_FILL, "install": _abi.REFRESH_INSTALL}[step]
+        check(lib().ugache_refresh_chunk(self.ctx, st, lo, hi, max_sms, _stream_handle(stream)),
+              "ugache_refresh_chunk", self.ctx)
+
     def refresh_commit(self, stream=None):
         check(lib().ugache_refresh_commit(self.ctx, _stream_handle(stream)), "ugache_refresh_commit",
               self.ctx)
+
+    def calibrate(self, sample_rows: int = 0) -> dict:
+        """A0 calibration through this ctx's sources (ugache_calibrate): bandwidth vs SMs for
+        the host and the peers, local gather bandwidth, and the recommended SM counts.  Call
+        on every rank at once for the contention of all G readers."""
+        c = _abi.ugache_calibration()
+        check(lib().ugache_calibrate(self.ctx, sample_rows, ctypes.byref(c)), "ugache_calibrate", self.ctx)
+        return {"host_sms": c.host_sms, "peer_sms": c.peer_sms, "bw_local": c.bw_local,
+                "bw_peer": c.bw_peer, "bw_host": c.bw_host, "sample_rows": c.sample_rows,
+                "host_curve": [(c.host_points_sms[i], c.host_points_bw[i]) for i in range(c.n_host_points)],
+                "peer_curve": [(c.peer_points_sms[i], c.peer_points_bw[i]) for i in range(c.n_peer_points)]}
 
     def set_dedication(self, host_sms: int = 0, peer_sms: int = 0):
         check(lib().ugache_set_dedication(self.ctx, host_sms, peer_sms), "ugache_set_dedication", self.ctx)
@@ -217,6 +253,11 @@ class UGache:
 
     def set_host_walk(self, on: bool):
         self.set_option(_abi.OPT_HOST_WALK, int(on))
+
+    def set_preorder(self, on: bool = True):
+        """UGACHE_OPT_PREORDER: host range histogram built while locating, host bucket ordered
+        by every CTA (default on)."""
+        self.set_option(_abi.OPT_PREORDER, int(on))
 
     def set_stage_host_io(self, on: bool):
         self.set_option(_abi.OPT_STAGE_HOST_IO, int(on))
@@ -276,8 +317,9 @@ class UGache:
         return n.value
 
     def last_batch_phases(self):
-        """(locate done, host ordered, host copies done) in ms from the fused kernel's start."""
-        ms = (ctypes.c_float * 3)()
+        """(locate done, host ordered, host copies done, last CTA located, launch end) in ms
+        from the fused kernel's start (ugache_last_batch_phases)."""
+        ms = (ctypes.c_float * 5)()
         check(lib().ugache_last_batch_phases(self.ctx, ms), "ugache_last_batch_phases", self.ctx)
         return tuple(float(x) for x in ms)
 

@@ -349,6 +349,64 @@ class HostTable:
             self._fd = None
 
 
+class AliasedHostTable:
+    """An N-row table whose virtual span is full size but whose physical memory is only the
+    first ``phys_rows`` rows: one memfd of phys_rows * R bytes mapped repeatedly at adjacent
+    addresses (MAP_FIXED inside one reserved range), so row k holds the generator's row
+    ``k mod phys_rows``.  Used to run full-size DLR / MAG key spaces (375-410 GB) on a box
+    with less RAM: the device sees the full host address span (translation footprint), and
+    the oracle reads the same buffer, so parity is unaffected.  Same interface as HostTable
+    (``ptr``, ``array`` over the whole span, ``fill``, ``close``)."""
+
+    def __init__(self, num_rows: int, row_bytes: int, phys_rows: int):
+        libc = ctypes.CDLL(None, use_errno=True)
+        libc.mmap.restype = ctypes.c_void_p
+        libc.mmap.argtypes = [ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int, ctypes.c_int,
+                              ctypes.c_int, ctypes.c_long]
+        libc.munmap.argtypes = [ctypes.c_void_p, ctypes.c_size_t]
+        self._libc = libc
+        self.num_rows, self.row_bytes = int(num_rows), int(row_bytes)
+        gran = 4096  # rows: phys_rows * R stays a multiple of 2 MB for 512-B multiples
+        self.phys_rows = max(gran, min(self.num_rows, (int(phys_rows) // gran) * gran))
+        self.nbytes = self.num_rows * self.row_bytes
+        self.phys_bytes = self.phys_rows * self.row_bytes
+        self.copies = -(-self.num_rows // self.phys_rows)
+        self.shm_path = None
+        self._fd = os.memfd_create("ugache_aliased_table")
+        os.ftruncate(self._fd, self.phys_bytes)
+        PROT_NONE, PROT_RW = 0, 3
+        MAP_SHARED, MAP_PRIVATE, MAP_FIXED, MAP_ANON, MAP_NORESERVE = 0x01, 0x02, 0x10, 0x20, 0x4000
+        total = self.copies * self.phys_bytes
+        base = libc.mmap(None, total, PROT_NONE, MAP_PRIVATE | MAP_ANON | MAP_NORESERVE, -1, 0)
+        if base in (None, ctypes.c_void_p(-1).value):
+            raise OSError(ctypes.get_errno(), "reserving the aliased table span failed")
+        self._base, self._total = base, total
+        for i in range(self.copies):
+            at = libc.mmap(base + i * self.phys_bytes, self.phys_bytes, PROT_RW,
+                           MAP_SHARED | MAP_FIXED, self._fd, 0)
+            if at != base + i * self.phys_bytes:
+                raise OSError(ctypes.get_errno(), f"mapping alias copy {i} failed")
+        buf = (ctypes.c_uint8 * self.nbytes).from_address(base)
+        self.array = np.frombuffer(buf, dtype=np.uint8, count=self.nbytes).reshape(self.num_rows, self.row_bytes)
+
+    @property
+    def ptr(self) -> int:
+        return int(self._base)
+
+    def fill(self, seed: int = TABLE_SEED):
+        """Generator rows 0..phys_rows-1 (every alias copy sees them)."""
+        _lib().synth_fill_table(ctypes.c_void_p(self._base), 0, self.phys_rows, self.row_bytes // 4, seed)
+
+    def close(self):
+        self.array = None
+        if self._base:
+            self._libc.munmap(ctypes.c_void_p(self._base), self._total)
+            self._base = 0
+        if self._fd is not None:
+            os.close(self._fd)
+            self._fd = None
+
+
 def make_table(num_rows: int, row_bytes: int, seed: int = TABLE_SEED) -> HostTable:
     t = HostTable(num_rows, row_bytes)
     t.fill(seed=seed)

@@ -36,7 +36,7 @@ def test_library_exports_every_declared_symbol():
 def test_struct_layouts_match_header():
     # sizes follow from the header's field list (no implicit padding surprises)
     assert ctypes.sizeof(_abi.ugache_config) == 8 + 4 + 4 + 8 + 4 * 4 + 8 * 3 + 4 * 4
-    assert ctypes.sizeof(_abi.ugache_plan) == 4 + 4 + 8 * 3 + 8 * 9 + 4 * 4
+    assert ctypes.sizeof(_abi.ugache_plan) == 4 + 4 + 8 * 3 + 8 * 9 + 4 * 4 + 8
 
 
 @pytest.mark.parametrize("field,value", [
@@ -182,9 +182,31 @@ def test_fill_host_tier_matches_generator():
     plan, order = solve(cfg, h)
     t = synth.make_table(N, R)
     rows = host_tier_rows(plan, N)
-    assert rows == N - plan.band_end
+    assert rows == N                       # every row: host-resident ranks first, then cached
     tier = np.empty((rows, R), dtype=np.uint8)
     fill_host_tier(cfg, order, plan, t, tier)
-    keys = order.astype(np.int64)[plan.band_end:]
+    keys = np.roll(order.astype(np.int64), -int(plan.band_end))     # slot t: rank (be + t) mod N
     assert np.array_equal(tier, synth.rows_for_keys(keys, N, R))
     t.close()
+
+
+@pytest.mark.parametrize("G,k_frac,alpha", [(1, 1.0, 1.2), (2, 0.5, 1.2), (4, 0.0, 0.9), (8, 0.3, 1.4)])
+def test_model_time_matches_oracle_model(G, k_frac, alpha):
+    """ugache_model_time (the Refresher's trigger model behind the ABI) equals the oracle's
+    section 6.2 model (oracle.placement.model_times) on family placements and on a shuffled
+    (arbitrary) placement, with the plan's T / R."""
+    from oracle.placement import Platform, model_times
+    from paper_conf_sosp_songz0c23_b200 import model_time
+    N, C = 4000, 300
+    h = _hot(N, alpha, "zipf")
+    cfg = make_config(N, 512, C, num_gpus=G, host_sms=8, bw_local=6457.7e9, bw_peer=770e9, bw_host=34.4e9)
+    plan, order = solve(cfg, h)
+    plat = Platform(G=G, row_bytes=512, bw_local=6457.7e9, bw_peer=770e9, bw_host=34.4e9, host_sms=8,
+                    peer_sms=int(plan.peer_sms), num_sms=int(plan.num_sms))
+    loc, _ = policy_placement(rank_order(h, N), N, C, G, int(k_frac * C))
+    z_ref, _, _ = model_times(h, loc, plat)
+    assert abs(model_time(plan, list(loc), h) - z_ref) <= 1e-9 * z_ref
+    rng = np.random.default_rng(G)
+    shuffled = np.stack([l[rng.permutation(N)] for l in loc])       # any table: only src counts
+    z_ref2, _, _ = model_times(h, shuffled, plat)
+    assert abs(model_time(plan, list(shuffled), h) - z_ref2) <= 1e-9 * z_ref2

@@ -1,5 +1,5 @@
 """Control plane over torch.distributed with the gloo backend, world size 2, on CPU:
-IPC-handle exchange with the placement digest, max/sum over ranks."""
+IPC-handle exchange with the placement digest, max/sum over ranks, per-rank row gather."""
 import os
 import socket
 
@@ -29,10 +29,11 @@ def _worker(rank, ws, port, q, same_digest):
         handles = ugd.exchange_handles(bytes([rank]) * 64, digest)
         mx = ugd.max_over_ranks(float(rank + 1))
         sm = ugd.sum_over_ranks(float(rank + 1))
+        rows = ugd.gather_rows([rank, 10.0 * rank + 1, -rank])
         ugd.barrier()
-        q.put((rank, [h[0] for h in handles], mx, sm, None))
+        q.put((rank, [h[0] for h in handles], mx, sm, rows.tolist(), None))
     except Exception as e:  # noqa: BLE001
-        q.put((rank, None, None, None, repr(e)))
+        q.put((rank, None, None, None, None, repr(e)))
     finally:
         dist.destroy_process_group()
 
@@ -52,12 +53,13 @@ def _run(same_digest):
 
 def test_handle_exchange_and_reductions_gloo_ws2():
     res = _run(True)
-    for rank, handles, mx, sm, err in res:
+    for rank, handles, mx, sm, rows, err in res:
         assert err is None, err
         assert handles == [0, 1]          # rank order
         assert mx == 2.0 and sm == 3.0
+        assert rows == [[0.0, 1.0, 0.0], [1.0, 11.0, -1.0]]   # every rank's row, rank order
 
 
 def test_placement_digest_mismatch_is_detected():
     res = _run(False)
-    assert all(err is not None and "different placements" in err for _, _, _, _, err in res)
+    assert all(err is not None and "different placements" in err for _, _, _, _, _, err in res)

@@ -617,7 +617,8 @@ def test_stream_auto_switches_on_host_density(torch_cuda):
     loc, _ = c.export_placement()
     host_keys = np.nonzero((loc >> 56) == 1)[0]
     local_keys = np.nonzero((loc >> 56) == 0)[0]
-    prev_dense = False
+    # before any launch the choice comes from the plan's expected host keys
+    prev_dense = 200_000 * c.plan.host_mass_frac >= 4096
     for b in range(7):
         dense = b in (2, 3, 4)
         keys = rng.choice(host_keys if dense else local_keys, 200_000)
@@ -708,8 +709,8 @@ def test_fused_phase_stamps(torch_cuda):
     keys = np.random.default_rng(55).integers(0, N, 200_000)   # ~97 % host keys: dense
     check_batch(torch_cuda, c, t, keys, N, R, 1)
     loc_ms, gat_ms = c.last_batch_timing()
-    a, b, d = c.last_batch_phases()
-    assert 0 < a <= b <= d <= (loc_ms + gat_ms) * 1.05 + 0.01
+    a, b, d, la, e = c.last_batch_phases()
+    assert 0 < la <= a <= b <= d <= e <= (loc_ms + gat_ms) * 1.05 + 0.01
     c.set_stream("on")
     check_batch(torch_cuda, c, t, keys[:5000], N, R, 1)
     with pytest.raises(UGacheError):
@@ -736,3 +737,201 @@ def test_single_pass_host_first_groups(torch_cuda, monkeypatch, group, sched):
             check_batch(torch_cuda, c, t, keys, N, R, G)
         for g in group_:
             g.close()
+
+
+@pytest.mark.parametrize("fused", ["on", "off"])
+@pytest.mark.parametrize("G,tier", [(1, False), (1, True), (2, False), (4, True)])
+def test_preorder_parity(torch_cuda, fused, G, tier):
+    """UGACHE_OPT_PREORDER: the host range histogram is built while locating and every CTA
+    scatters a slice of the host bucket; bit-exact against the oracle and against the host
+    CTAs' own ordering, on the fused and split paths, with and without the host tier, and
+    across dense -> sparse -> dense launches (the histogram is re-armed either way)."""
+    N, R = 300_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(60).permutation(N)]
+    t, group = make_group(torch_cuda, N, R, 4000, G, h, host_tier=tier)
+    rng = np.random.default_rng(61)
+    for g, c in enumerate(group):
+        c.set_stream("off")
+        c.set_fused(fused)
+        for pre in (True, False, True):
+            c.set_preorder(pre)
+            for n, dense in ((150_000, True), (3_000, False), (120_001, True)):
+                keys = rng.integers(-3, N + 3, n)
+                per = check_batch(torch_cuda, c, t, keys, N, R, G)
+                assert (per[G] >= 4096) == dense
+    for c in group:
+        c.close()
+
+
+def test_preorder_phase_stamps(torch_cuda):
+    """With pre-ordering, host copies begin right after the locate boundary: the host bucket
+    is ordered before the copies start, every stamp is inside the launch."""
+    N, R = 300_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(62).permutation(N)]
+    t, (c,) = make_group(torch_cuda, N, R, 10_000, 1, h, host_tier=True)
+    c.enable_timing(True)
+    c.set_stream("off")
+    c.set_fused("on")
+    keys = np.random.default_rng(63).integers(0, N, 200_000)
+    for _ in range(3):
+        check_batch(torch_cuda, c, t, keys, N, R, 1)
+        loc_ms, gat_ms = c.last_batch_timing()
+        located, ordered, host_done, last_loc, end = c.last_batch_phases()
+        assert 0 < last_loc <= located <= ordered <= host_done <= end <= (loc_ms + gat_ms) * 1.05 + 0.01
+    c.close()
+
+
+def test_first_batch_path_from_plan(torch_cuda):
+    """UGACHE_OPT_STREAM = auto before any launch: the path follows the plan's expected host
+    keys (n x host_mass_frac vs the ordering threshold), not a default."""
+    N, R = 400_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(64).permutation(N)]
+    for C, n in ((8_000, 200_000), (300_000, 20_000)):
+        t, (c,) = make_group(torch_cuda, N, R, C, 1, h)
+        expect_dense = n * c.plan.host_mass_frac >= 4096
+        assert expect_dense == (C == 8_000)
+        keys = np.random.default_rng(65).choice(N, n, p=h / h.sum())
+        check_batch(torch_cuda, c, t, keys, N, R, 1)
+        assert c.last_extract_path() == ("fused" if expect_dense else "single_pass")
+        c.close()
+
+
+@pytest.mark.parametrize("inline", ["host", "none"])
+def test_fresh_ctx_on_nonblocking_stream(torch_cuda, inline):
+    """The scratch (queue sentinels, sub-queue counters) of a fresh ctx is initialised on the
+    extract stream: the first launches on a non-blocking stream are bit-exact, including
+    queued host rows (inline none) and a batch that grows the scratch."""
+    N, R = 200_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(66).permutation(N)]
+    t, (c,) = make_group(torch_cuda, N, R, 20_000, 1, h)
+    c.set_stream("on")
+    c.set_inline(host=inline == "host", peers=False)
+    s = torch_cuda.cuda.Stream()
+    for n in (30_000, 250_000):
+        keys_np = np.random.default_rng(n).integers(0, N, n)
+        keys = torch_cuda.from_numpy(keys_np).cuda()
+        torch_cuda.cuda.synchronize()
+        out = torch_cuda.empty((n, R), dtype=torch_cuda.uint8, device="cuda")
+        c.extract(keys, out, s)
+        s.synchronize()
+        ref, _ = oracle.gather(t.ptr, N, R, keys_np)
+        assert np.array_equal(out.cpu().numpy(), ref)
+    c.close()
+
+
+def test_init_rejects_bad_order_plan_and_alignment(torch_cuda):
+    """ugache_init_with_plan: an order that is not a permutation, or a plan larger than the
+    config's capacity, is EINVAL; a host table that is not 16-byte aligned is EINVAL (the
+    kernels read rows with 16-byte vector loads and bulk copies)."""
+    from paper_conf_sosp_songz0c23_b200 import UGache, make_config, solve
+    from paper_conf_sosp_songz0c23_b200._abi import UGACHE_EINVAL, UGacheError
+    N, R, C = 20_000, 512, 1000
+    t = table_for(N, R)
+    h = (synth.zipf_pmf(N, 1.2) * 1e4).astype(np.float32)
+    cfg = make_config(N, R, C, host_tier=True)
+    plan, order = solve(cfg, h)
+    bad = order.copy()
+    bad[5] = bad[6]                                   # duplicate key, one key missing
+    with pytest.raises(UGacheError) as e:
+        UGache(t, N, R, C, plan=plan, order=bad, host_tier=True)
+    assert e.value.status == UGACHE_EINVAL
+    big_cfg = make_config(N, R, 2 * C)
+    big_plan, big_order = solve(big_cfg, h)
+    with pytest.raises(UGacheError) as e:
+        UGache(t, N, R, C, plan=big_plan, order=big_order)
+    assert e.value.status == UGACHE_EINVAL
+    raw = np.empty(N * R + 16, dtype=np.uint8)
+    off = (-raw.ctypes.data) % 16 + 8                 # 8 bytes past a 16-byte boundary
+    mis = raw[off: off + N * R]
+    with pytest.raises(UGacheError) as e:
+        UGache(mis, N, R, C, hotness=h)
+    assert e.value.status == UGACHE_EINVAL
+    ok = UGache(t, N, R, C, plan=plan, order=order, host_tier=True)   # the valid pair works
+    ok.fill()
+    check_batch(torch_cuda, ok, t, np.arange(0, N, 7), N, R, 1)
+    ok.close()
+
+
+@pytest.mark.parametrize("protocol", ["chunked", "whole"])
+@pytest.mark.parametrize("G", [1, 3])
+def test_cache_refresh_with_host_tier(torch_cuda, protocol, G):
+    """Section 7.2 refresh on a host-tier ctx (the shipped configuration): keys evicted from
+    the cache are redirected to their slot of the tier (which holds every row), extraction
+    stays bit-exact through every step of the chunked (stage / evict / fill / install per
+    slot range) and whole-table (begin / content / commit) protocols, and the committed table
+    equals the new placement with host rows mapped to tier slots."""
+    from paper_conf_sosp_songz0c23_b200 import UGache, connect_in_process, make_config, solve
+    from paper_conf_sosp_songz0c23_b200.refresh import plan_placements, refresh_group
+    N, R, C = 120_000, 512, 7000
+    p = (synth.zipf_pmf(N, 1.2) * 8192).astype(np.float32)
+    h1 = p[np.random.default_rng(71).permutation(N)]
+    h2 = p[np.random.default_rng(72).permutation(N)]
+    t = table_for(N, R)
+    group = [UGache(t, N, R, C, hotness=h1, num_gpus=G, rank=g, host_tier=True) for g in range(G)]
+    connect_in_process(group)
+    for c in group:
+        c.fill()
+    plan1, order1 = solve(make_config(N, R, C, num_gpus=G, host_tier=True), h1)
+    be1 = int(plan1.band_end)
+    tier_slot = np.empty(N, dtype=np.uint64)
+    tier_slot[order1.astype(np.int64)] = (np.arange(N, dtype=np.uint64) + np.uint64(N - be1)) % np.uint64(N)
+    _, pl2 = plan_placements(dict(num_rows=N, row_bytes=R, capacity_rows=C), h2, G)
+    rng = np.random.default_rng(73)
+    cdf = np.cumsum(h2.astype(np.float64)) / h2.sum()
+    batches = [np.searchsorted(cdf, rng.random(30_000)).astype(np.int64) for _ in range(G)]
+    n_fg = [0]
+
+    def foreground():
+        for g, c in enumerate(group):
+            check_batch(torch_cuda, c, t, batches[g], N, R, G)
+        n_fg[0] += 1
+
+    foreground()
+    if protocol == "chunked":
+        refresh_group(group, pl2, max_sms=4, max_rows=2000, foreground=foreground)
+        assert n_fg[0] >= 1 + (C + 1999) // 2000
+    else:
+        for c, (loc, sk) in zip(group, pl2):
+            c.refresh_begin(loc, sk)
+        foreground()
+        for c in group:
+            while c.refresh_content(max_sms=4, max_rows=3000) > 0:
+                foreground()
+        torch_cuda.cuda.synchronize()
+        foreground()
+        for c in group:
+            c.refresh_commit()
+    foreground()
+    host = np.uint64(G) << np.uint64(56)
+    for g, c in enumerate(group):
+        loc, sk = c.export_placement()
+        want = pl2[g][0].copy()
+        is_host = (want >> np.uint64(56)) == np.uint64(G)
+        want[is_host] = host | tier_slot[is_host]
+        assert np.array_equal(loc, want) and np.array_equal(sk, pl2[g][1])
+    for c in group:
+        c.close()
+
+
+@pytest.mark.parametrize("G", [1, 2])
+def test_calibrate(torch_cuda, G):
+    """ugache_calibrate (A0): host bandwidth vs SMs over the swept counts, the recommended
+    host SMs is the first point within 90 % of the best, local gather beats the host link,
+    and with peers the all-to-all ingress curve is measured; extraction is unaffected."""
+    N, R = 400_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(81).permutation(N)]
+    t, group = make_group(torch_cuda, N, R, 20_000, G, h, host_tier=True)
+    cal = group[0].calibrate(16384)
+    ks = [k for k, _ in cal["host_curve"]]
+    bws = [b for _, b in cal["host_curve"]]
+    assert ks == sorted(ks) and ks[0] == 1 and len(ks) >= 8 and all(b > 0 for b in bws)
+    first90 = next(k for k, b in cal["host_curve"] if b >= 0.9 * max(bws))
+    assert cal["host_sms"] == first90 and cal["bw_host"] >= 0.9 * max(bws)
+    assert cal["bw_local"] > cal["bw_host"] and cal["sample_rows"] == 16384
+    if G > 1:
+        assert cal["peer_curve"] and cal["peer_sms"] >= 1 and cal["bw_peer"] > 0
+    else:
+        assert cal["peer_curve"] == [] and cal["peer_sms"] == 0
+    check_batch(torch_cuda, group[0], t, np.random.default_rng(82).integers(0, N, 50_000), N, R, G)
+    for c in group:
+        c.close()

@@ -116,3 +116,18 @@ def test_hotness_orders_by_rank():
     hr[ranks] = h
     assert np.all(np.diff(hr.astype(np.float64)) <= 0)
     assert abs(h.sum() - 8192) < 1.0
+
+
+def test_aliased_table_rows_repeat_the_physical_prefix():
+    """AliasedHostTable: a full-size span backed by phys_rows physical rows mapped repeatedly;
+    row k is the generator's row k mod phys_rows, writes through one alias show in all."""
+    N, R, P = 20_000, 512, 4096
+    t = synth.AliasedHostTable(N, R, P)
+    t.fill()
+    assert t.phys_rows == P and t.copies == 5 and t.array.shape == (N, R)
+    keys = np.array([0, 1, P - 1, P, P + 7, 3 * P + 11, N - 1])
+    want = synth.rows_for_keys(keys % P, N, R)
+    assert np.array_equal(t.array[keys], want)
+    t.array[5, :4] = 7                     # shared physical page
+    assert np.all(t.array[P + 5, :4] == 7) and np.all(t.array[4 * P + 5, :4] == 7)
+    t.close()
