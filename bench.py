@@ -671,11 +671,13 @@ def main():
     traffic = traffic_pcie = traffic_src = None
     try:  # per-launch DRAM traffic of the kernel from the committed ncu capture of this config
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
-            rec = json.load(f)[wl.name][kname]
+            recs = json.load(f)[wl.name][kname]
         c_run = args.cache_ratio if args.cache_ratio is not None else wl.cache_ratio
-        if (abs(rec.get("cache_ratio", wl.cache_ratio) - c_run) < 1e-9 and
-                bool(rec.get("host_tier", False)) == bool(args.host_tier) and rec.get("n_gpus", 1) == ws):
-            traffic, traffic_pcie, traffic_src = rec["dram_bytes"], rec.get("pcie_read_bytes"), rec["source"]
+        for rec in (recs if isinstance(recs, list) else [recs]):
+            if (abs(rec.get("cache_ratio", wl.cache_ratio) - c_run) < 1e-9 and
+                    bool(rec.get("host_tier", False)) == bool(args.host_tier) and rec.get("n_gpus", 1) == ws):
+                traffic, traffic_pcie, traffic_src = rec["dram_bytes"], rec.get("pcie_read_bytes"), rec["source"]
+                break
     except Exception:
         pass
     # duplicate-aware variant: source reads counted per unique row of the

@@ -339,7 +339,7 @@ ugache_status ugache_set_mode(ugache_ctx *ctx, int32_t mode);
  *    in that order; 0 = copy in bucket order.
  *  UGACHE_OPT_STAGE_HOST_IO (default 0): 1 = stage pinned host keys/out through device
  *    buffers + cudaMemcpyAsync instead of zero-copy access from the kernels.
- *  UGACHE_OPT_HOST_WARPS (default 8, 1..16): warps per host CTA that read host rows; the
+ *  UGACHE_OPT_HOST_WARPS (default 12, 1..16): warps per host CTA that read host rows; the
  *    others pad local work (A0 calibration knob).
  *  UGACHE_OPT_DEDICATION: UGACHE_DEDICATE_SMS = the paper's core dedication, whole SMs per
  *    source; UGACHE_DEDICATE_WARPS = the same dedication at warp granularity:
@@ -452,6 +452,8 @@ ugache_status ugache_read_slab(ugache_ctx *ctx, uint64_t first, uint64_t count, 
 ugache_status ugache_destroy(ugache_ctx *ctx);
 
 const char *ugache_error_string(ugache_status st);
+/* Detail text of the ctx's last error (CUDA error name and call, ...); with ctx == NULL,
+ * the detail of the calling thread's last failed ugache_init* (the ctx is gone). */
 const char *ugache_last_error_message(const ugache_ctx *ctx);
 int32_t ugache_version(void);
 

@@ -31,7 +31,7 @@ constexpr int kGatherThreads = 512;  // 16 warps; one CTA per SM (forced via sme
 constexpr int kGatherWarps = kGatherThreads / 32;
 constexpr int kRowsInFlight = 8;     // rows per warp per step (U)
 constexpr int kLocalChunk = 64;      // rows per local-cursor claim
-constexpr int kHostWarps = 8;        // warps per host CTA reading host rows (A0 calibration)
+constexpr int kHostWarps = 12;       // warps per host CTA reading host rows (A0 calibration, round 2)
 constexpr uint32_t kFullMask = 0xFFFFFFFFu;
 constexpr int kMaxSmId = 256;        // role table size, indexed by %smid
 

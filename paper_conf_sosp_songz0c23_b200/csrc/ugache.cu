@@ -448,6 +448,9 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_HOST_ROWS")) ctx->host_rows = atoi(e);
   if (const char *e = getenv("UGACHE_EARLY_WALK")) ctx->early_walk = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_PREORDER")) ctx->preorder = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_L2_FETCH")) {  // experiment: device-wide L2 fetch granularity
+    UG_CUDA(ctx, cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, (size_t)atoi(e)));
+  }
   if (const char *e = getenv("UGACHE_HIST_SMEM")) ctx->hist_smem = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_HOST_SEGMENTS")) ctx->host_segments = std::max(1, std::min(8, atoi(e)));
   if (const char *e = getenv("UGACHE_LOCAL_BULK")) ctx->local_bulk = std::max(0, std::min(3, atoi(e)));
@@ -538,8 +541,12 @@ const char *ugache_error_string(ugache_status st) {
   return "unknown status";
 }
 
+namespace {
+thread_local std::string g_init_err;  // detail of this thread's last failed init
+}
+
 const char *ugache_last_error_message(const ugache_ctx *ctx) {
-  return ctx ? ctx->err.c_str() : "";
+  return ctx ? ctx->err.c_str() : g_init_err.c_str();
 }
 
 static ugache_status init_impl(ugache_ctx **out, const ugache_config *cfg, const void *host_table,
@@ -616,6 +623,7 @@ static ugache_status init_impl(ugache_ctx **out, const ugache_config *cfg, const
   if (st == UGACHE_OK)
     st = init_common(ctx, cfg, host_table, order, host_tier, given_loc, given_slots, given_n);
   if (st != UGACHE_OK) {
+    g_init_err = ctx->err;
     ugache_destroy(ctx);
     return st;
   }
@@ -983,8 +991,9 @@ ugache_status ugache_calibrate(ugache_ctx *ctx, uint32_t sample_rows, ugache_cal
     if (e0) cudaEventDestroy(e0);
     if (e1) cudaEventDestroy(e1);
   };
-  cudaError_t ce = cudaMalloc(&d_ents, (size_t)roles_max * n * sizeof(uint64_t));
-  if (ce == cudaSuccess) ce = cudaMalloc(&d_out, (size_t)roles_max * n * R);
+  cudaError_t ce = cudaMalloc(&d_ents, (size_t)std::max(roles_max, 8) * n * sizeof(uint64_t));
+  const uint32_t n_local = n * 8;  // the local gather needs a larger sample to outlast the launch
+  if (ce == cudaSuccess) ce = cudaMalloc(&d_out, (size_t)std::max<uint64_t>((uint64_t)roles_max * n, n_local) * R);
   if (ce == cudaSuccess) ce = cudaMalloc(&d_flush, flush_bytes);
   if (ce == cudaSuccess) ce = cudaMalloc(&d_cursor, ugk::kMaxSrc * sizeof(uint32_t));
   if (ce == cudaSuccess) ce = cudaEventCreate(&e0);
@@ -1017,7 +1026,7 @@ ugache_status ugache_calibrate(ugache_ctx *ctx, uint32_t sample_rows, ugache_cal
       if (e != cudaSuccess) return e;
     }
     std::sort(ms, ms + 3);
-    *bw = (double)n_roles * n * R / (ms[1] * 1e-3);
+    *bw = (double)n_roles * cp.n_ents * R / (ms[1] * 1e-3);
     return cudaSuccess;
   };
   std::vector<uint64_t> ents;
@@ -1042,10 +1051,12 @@ ugache_status ugache_calibrate(ugache_ctx *ctx, uint32_t sample_rows, ugache_cal
   // local slab: every SM
   if (ce == cudaSuccess) {
     ents.clear();
-    calib_sample(ents, std::max<uint64_t>(ctx->n_slots, 1), n, seed++);
+    calib_sample(ents, std::max<uint64_t>(ctx->n_slots, 1), n_local, seed++);
     ce = cudaMemcpy(d_ents, ents.data(), ents.size() * 8, cudaMemcpyHostToDevice);
     cp.src_id[0] = me;
+    cp.n_ents = n_local;
     if (ce == cudaSuccess) ce = run(S, 1, &out->bw_local);
+    cp.n_ents = n;
   }
   // peers: all at once, k SMs per peer (all-to-all ingress)
   if (ce == cudaSuccess && G > 1) {

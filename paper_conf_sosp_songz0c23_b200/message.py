@@ -111,27 +111,40 @@ def message_extract_group(caches: Sequence[UGache], keys_list: Sequence, outs: S
 
 def message_extract(c: UGache, keys, out=None, group=None, stream=None):
     """One message-based batch on this rank; every rank of ``group`` calls it together.
-    Exchanges: all_to_all_single of counts, of slot ids, and of rows (NCCL)."""
+    Exchanges: all_to_all_single of counts, of slot ids, and of rows -- NCCL on device
+    buffers, or staged through host memory when the group's backend is gloo (ranks sharing
+    one GPU in tests)."""
     import torch
     import torch.distributed as dist
     G, me, R = c.num_gpus, c.rank, c.row_bytes
     if out is None:
         out = torch.empty((keys.numel(), R), dtype=torch.uint8, device="cuda")
+    host_xchg = dist.get_backend(group) == "gloo"
+
+    def a2a(dst, src, out_split=None, in_split=None):
+        if host_xchg:
+            d = torch.empty(dst.shape, dtype=dst.dtype)
+            torch.cuda.synchronize()
+            dist.all_to_all_single(d, src.cpu(), output_split_sizes=out_split,
+                                   input_split_sizes=in_split, group=group)
+            dst.copy_(d)
+        else:
+            dist.all_to_all_single(dst, src, output_split_sizes=out_split,
+                                   input_split_sizes=in_split, group=group)
+
     c._msg_n = keys.numel()
     _local(c, keys, out, stream)
     counts, req = _requests(c, stream)
     send_counts = [0 if j == me else int(counts[j]) for j in range(G)]
     sc = torch.tensor(send_counts, dtype=torch.int64, device="cuda")
     rc = torch.empty_like(sc)
-    dist.all_to_all_single(rc, sc, group=group)
+    a2a(rc, sc)
     recv_counts = rc.cpu().tolist()
     req_in = torch.empty(sum(recv_counts), dtype=torch.int32, device="cuda")
-    dist.all_to_all_single(req_in, req, output_split_sizes=recv_counts,
-                           input_split_sizes=send_counts, group=group)
+    a2a(req_in, req[: sum(send_counts)], recv_counts, send_counts)
     send = torch.empty((max(1, req_in.numel()), R), dtype=torch.uint8, device="cuda")
     _serve(c, req_in, send, stream)
-    rep = torch.empty((req.numel(), R), dtype=torch.uint8, device="cuda")
-    dist.all_to_all_single(rep, send[: req_in.numel()], output_split_sizes=send_counts,
-                           input_split_sizes=recv_counts, group=group)
+    rep = torch.empty((sum(send_counts), R), dtype=torch.uint8, device="cuda")
+    a2a(rep, send[: req_in.numel()], send_counts, recv_counts)
     _scatter(c, rep, out, stream)
     return out

@@ -128,7 +128,9 @@ class UGache:
             h = None if hotness is None else np.ascontiguousarray(hotness, dtype=np.float32)
             st = lib().ugache_init(ctypes.byref(self.ctx), ctypes.byref(self.cfg), _ptr(table),
                                    _ptr(h))
-        check(st, "ugache_init")
+        if st != _abi.UGACHE_OK:
+            m = lib().ugache_last_error_message(None)
+            raise _abi.UGacheError(st, "ugache_init", m.decode() if m else "")
         self.num_gpus, self.rank = num_gpus, rank
         self.row_bytes = row_bytes
         self.num_rows = num_rows

@@ -1,7 +1,9 @@
 """Multi-process peer path with real CUDA IPC: two processes (ranks of a G = 2 group) on
 one B200, each with its own context and cache slab, exchanging cudaIpcMemHandles over a
 gloo process group (ugache_ipc_handle / ugache_open_peers), sharing one /dev/shm host
-table; each rank's extraction is compared byte for byte with the oracle."""
+table; each rank's extraction is compared byte for byte with the oracle -- factored
+extraction, the message-based baseline over the process group, and a chunked cache
+refresh driven across the two processes."""
 import os
 import socket
 
@@ -57,6 +59,34 @@ def _worker(rank, ws, port, shm, q):
             cnt, _ = source_counts(loc, keys, wl.num_rows, ws)
             res.append((bool(np.array_equal(out.cpu().numpy(), ref)),
                         bool(np.array_equal(per, cnt)), int(per[1 - rank])))
+        # the message-based baseline over the real process group (all-to-alls staged through
+        # host memory on gloo), same batch, same placement
+        from paper_conf_sosp_songz0c23_b200.message import message_extract
+        keys = synth.make_batch(wl, rank, 0)
+        out = message_extract(cache, torch.from_numpy(keys).cuda())
+        torch.cuda.synchronize()
+        ref, _ = oracle.gather(table.ptr, wl.num_rows, wl.row_bytes, keys)
+        msg_ok = bool(np.array_equal(out.cpu().numpy(), ref))
+        # chunked refresh across the two processes (barriers between the steps), to a
+        # placement solved for a permuted hotness; extraction stays bit-exact throughout
+        from paper_conf_sosp_songz0c23_b200.refresh import plan_placements, refresh_distributed
+        h2 = h[np.random.default_rng(5).permutation(len(h))]
+        _, pl2 = plan_placements(dict(num_rows=wl.num_rows, row_bytes=wl.row_bytes,
+                                      capacity_rows=wl.capacity_rows), h2, ws)
+        fg_ok = []
+
+        def foreground():
+            k2 = synth.make_batch(wl, rank, 7)
+            o2 = cache.extract(torch.from_numpy(k2).cuda())
+            torch.cuda.synchronize()
+            r2, _ = oracle.gather(table.ptr, wl.num_rows, wl.row_bytes, k2)
+            fg_ok.append(bool(np.array_equal(o2.cpu().numpy(), r2)))
+
+        refresh_distributed(cache, pl2[rank], max_sms=4, max_rows=3000, foreground=foreground)
+        foreground()
+        loc2, sk2 = cache.export_placement()
+        refreshed = bool(np.array_equal(loc2, pl2[rank][0]) and np.array_equal(sk2, pl2[rank][1]))
+        res.append((msg_ok and all(fg_ok) and len(fg_ok) >= 3 and refreshed, True, 1))
         ugd.barrier()                      # peers stay mapped until everyone is done
         cache.close()
         q.put((rank, res, None))

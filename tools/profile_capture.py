@@ -7,6 +7,7 @@ captures of the 57 GB pinned host tier OOM-killed in round 1).
   --what traffic : the bench.py workload (host tier on by default), W warm-up + K timed
                    extracts of distinct batches, 256 MiB L2 flush before each -- the per-launch
                    DRAM / PCIe bytes of the dominant kernel (profiles/traffic.json).
+  --what calibrate : ugache_calibrate (A0) through the ctx of this workload.
   --what fig13   : Fig. 13 analog: the locally hit keys of one batch removed,
                    the remaining host keys extracted by the factored kernel and by random
                    dispatch (same placement), one warm-up + one measured launch each, L2
@@ -29,7 +30,7 @@ import numpy as np  # noqa: E402
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--what", default="traffic", choices=["traffic", "fig13"])
+    ap.add_argument("--what", default="traffic", choices=["traffic", "fig13", "calibrate"])
     ap.add_argument("--workload", default="gnn_pa")
     ap.add_argument("--cache-ratio", type=float, default=None)
     ap.add_argument("--no-host-tier", dest="host_tier", action="store_false", default=True)
@@ -71,7 +72,9 @@ def main():
         return s.elapsed_time(e)
 
     res = {"what": args.what, "workload": wl.name, "cache_ratio": wl.cache_ratio, "host_tier": args.host_tier}
-    if args.what == "traffic":
+    if args.what == "calibrate":
+        res["calibration"] = cache.calibrate()
+    elif args.what == "traffic":
         ms = [run(batches[i], out) for i in range(nb)]
         per, _ = cache.last_batch_stats()
         res.update(ms=ms[args.warmup:], path=cache.last_extract_path(), per_source=per.tolist())
@@ -82,6 +85,7 @@ def main():
         del loc
         dk = torch.from_numpy(np.ascontiguousarray(hk)).cuda()
         ho = torch.empty((len(hk), R), dtype=torch.uint8, device="cuda")
+        cache.set_stream("off")                                 # the two-phase factored kernel
         for mode in ("factored", "random"):
             cache.set_mode(mode)
             run(dk, ho)                                         # warm-up (the skipped launch)
