@@ -112,6 +112,10 @@ def parse():
                     help="full-size key span on a smaller box: back the N-row host table with this "
                          "many GB of physical rows mapped repeatedly (synth.AliasedHostTable); the "
                          "host tier is then off (it would need the full span physically)")
+    ap.add_argument("--calibrate", dest="calibrate", action="store_true", default=True,
+                    help="run ugache_calibrate (A0) on every rank at once before timing and report "
+                         "the curves in the JSON line (default)")
+    ap.add_argument("--no-calibrate", dest="calibrate", action="store_false")
     ap.add_argument("--print-world", action="store_true",
                     help="print this rank's RANK/WORLD_SIZE as JSON and exit (launch check)")
     return ap.parse_args()
@@ -240,6 +244,39 @@ def mem_available() -> int:
     except OSError:
         pass
     return 0
+
+
+def pin_alias_copies(table):
+    """Page-lock an AliasedHostTable copy by copy (the driver refuses one cudaHostRegister
+    over a span that maps the same physical pages twice) and check that every copy's device
+    address is its host address (UVA), so the library -- which uses already-pinned memory as
+    is -- reaches the whole span through the base pointer.  Returns the unpin function."""
+    import ctypes
+    rt = ctypes.CDLL("libcudart.so.12")
+    rt.cudaHostRegister.argtypes = [ctypes.c_void_p, ctypes.c_size_t, ctypes.c_uint]
+    rt.cudaHostUnregister.argtypes = [ctypes.c_void_p]
+    rt.cudaHostGetDevicePointer.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint]
+    done = []
+    for i in range(table.copies):
+        p = table.ptr + i * table.phys_bytes
+        n = min(table.phys_bytes, table.ptr + table.nbytes - p)
+        st = rt.cudaHostRegister(p, n, 1 | 2 | 8)          # portable | mapped | read-only
+        if st:
+            rt.cudaGetLastError()
+            st = rt.cudaHostRegister(p, n, 1 | 2)
+        if st:
+            raise RuntimeError(f"cudaHostRegister of alias copy {i} failed: {st}")
+        done.append(p)
+        d = ctypes.c_void_p()
+        rt.cudaHostGetDevicePointer(ctypes.byref(d), p, 0)
+        if d.value != p:
+            raise RuntimeError("registered host memory is not identity-mapped (UVA); aliased spans "
+                               "cannot be presented to the device as one range")
+
+    def unpin():
+        for p in done:
+            rt.cudaHostUnregister(p)
+    return unpin
 
 
 def setup_table(wl, rank, ws, torch_dist, alias_gb=0.0):
@@ -382,9 +419,10 @@ def main():
     dev_idx = local % ndev
     torch.cuda.set_device(dev_idx)
     dev = torch.device("cuda", dev_idx)
-    if ws > 1:
-        # NCCL when every rank owns a GPU (the normal case); gloo only for the control plane
-        # when ranks share a device (a functional multi-rank run on a 1-GPU box).
+    if ws > 1 or ("MASTER_ADDR" in os.environ and "WORLD_SIZE" in os.environ):
+        # NCCL when every rank owns a GPU (the normal case, also a 1-rank torchrun launch);
+        # gloo only for the control plane when ranks share a device (a functional multi-rank
+        # run on a 1-GPU box).
         if ndev >= ws:
             tdist.init_process_group("nccl", device_id=dev)
         else:
@@ -401,6 +439,7 @@ def main():
         log("host tier off: it needs another full copy of the table in host RAM")
         args.host_tier = False
     table = setup_table(wl, rank, ws, tdist, args.alias_gb)
+    unpin_alias = pin_alias_copies(table) if isinstance(table, synth.AliasedHostTable) else None
     t0 = time.time()
     h = synth.hotness(wl)
     log(f"hotness in {time.time() - t0:.1f}s")
@@ -437,6 +476,20 @@ def main():
     stream.synchronize()
     ugdist.barrier()
     log(f"fill in {time.time() - t0:.2f}s")
+    calibration = None
+    if args.calibrate:
+        # A0 (ugache_calibrate) on every rank at the same time: the host link and each GPU's
+        # NVLink egress carry the load of all G readers.  Reported, not applied:
+        # the shipped dedication is the workload calibration.
+        ugdist.barrier()
+        t0 = time.time()
+        cal = cache.calibrate()
+        calibration = {k: v for k, v in cal.items()}
+        calibration["host_curve_gbs"] = [(k_, b / 1e9) for k_, b in cal["host_curve"]]
+        calibration["peer_curve_gbs"] = [(k_, b / 1e9) for k_, b in cal["peer_curve"]]
+        del calibration["host_curve"], calibration["peer_curve"]
+        log(f"calibration in {time.time() - t0:.2f}s: host_sms {cal['host_sms']} "
+            f"({cal['bw_host'] / 1e9:.1f} GB/s), peer_sms {cal['peer_sms']}")
     if args.mode == "random":
         cache.set_mode("random")
     cache.set_stream(args.stream)
@@ -758,6 +811,7 @@ def main():
         "gpu_launches": int(ugdist.sum_over_ranks(float(launches))),
         "clocks": clk,
         "parity": parity,
+        "calibration": calibration,
         "plan": {"k": plan.k, "band_end": plan.band_end, "capacity_rows": plan.capacity_rows,
                  "host_sms": plan.host_sms, "peer_sms": plan.peer_sms,
                  "z_model_us": plan.z * 1e6, "z_replication_us": plan.z_replication * 1e6,
@@ -787,13 +841,15 @@ def main():
         print(json.dumps(line), flush=True)
     cache.close()
     ugdist.barrier()
+    if unpin_alias:
+        unpin_alias()
     for buf in (table, tier):
         if isinstance(buf, (synth.HostTable, synth.AliasedHostTable)):
             path = buf.shm_path
             buf.close()
             if ws > 1 and rank == 0 and path and os.path.exists(path):
                 os.unlink(path)
-    if ws > 1:
+    if tdist.is_initialized():
         tdist.destroy_process_group()
 
 

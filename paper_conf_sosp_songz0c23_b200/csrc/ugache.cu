@@ -448,9 +448,7 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_HOST_ROWS")) ctx->host_rows = atoi(e);
   if (const char *e = getenv("UGACHE_EARLY_WALK")) ctx->early_walk = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_PREORDER")) ctx->preorder = atoi(e) != 0;
-  if (const char *e = getenv("UGACHE_L2_FETCH")) {  // experiment: device-wide L2 fetch granularity
-    UG_CUDA(ctx, cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, (size_t)atoi(e)));
-  }
+
   if (const char *e = getenv("UGACHE_HIST_SMEM")) ctx->hist_smem = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_HOST_SEGMENTS")) ctx->host_segments = std::max(1, std::min(8, atoi(e)));
   if (const char *e = getenv("UGACHE_LOCAL_BULK")) ctx->local_bulk = std::max(0, std::min(3, atoi(e)));

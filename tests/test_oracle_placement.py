@@ -240,3 +240,28 @@ def test_host_tier_worked_example():
         check_placement(loc, sk, N, C, tier_keys=tier[::-1])
     with pytest.raises(AssertionError):
         check_placement(loc, sk, N, C)           # host rows are not keys any more
+
+
+def test_tiny_source_mix_matches_closed_form_coverage():
+    """SURVEY.md 8(c) source-mix sanity: batch means of the per-source key shares on tiny
+    (N = 100K, C = 10K per GPU, Zipf(1.2), 8,192 i.i.d. keys) match the closed-form Zipf
+    coverage: replication local 94.26 % / host 5.74 %; partition over G = 2 local 48.1 %,
+    peer 48.1 %, host 3.73 % (the mean over both GPUs).  Sampled through synth's batches and
+    the oracle's placement + source counts, so a wrong rank->key map, placement or count fails."""
+    wl = synth.get_workload("tiny")
+    N, C, G = wl.num_rows, wl.capacity_rows, 2
+    order = rank_order(synth.hotness(wl), N)
+    shares = {}
+    for name, k in (("replication", C), ("partition", 0)):
+        loc, _ = policy_placement(order, N, C, G, k)
+        tot = np.zeros(3)
+        for g in range(G):
+            for b in range(10):
+                keys = synth.make_batch(wl, g, b)
+                cnt, _ = source_counts(loc[g], keys, N, G)
+                tot += [cnt[g], cnt[1 - g], cnt[G]]
+        shares[name] = tot / tot.sum()
+    rep, part = shares["replication"], shares["partition"]
+    assert abs(rep[0] - 0.9426) < 0.004 and rep[1] == 0 and abs(rep[2] - 0.0574) < 0.004
+    assert abs(part[0] - 0.481) < 0.006 and abs(part[1] - 0.481) < 0.006
+    assert abs(part[2] - 0.0373) < 0.004
