@@ -761,6 +761,12 @@ def main():
                      "kernel": kname + {"fused": " (K1 locate+bucket and K2 gather, one cooperative launch)",
                                         "single_pass": " (K3: locate + copy in one pass, no grid barrier)"}.get(path, ""),
                      "path": path, "rank": slow,
+                     "random_row_peak": ({"peak": max(b for _, b in calibration["host_curve_gbs"]),
+                                          "frac": achieved / max(b for _, b in calibration["host_curve_gbs"]),
+                                          "source": "ugache_calibrate this run: best of the host-source "
+                                                    "curve (sorted uniform random rows, k SMs swept)"}
+                                         if bound == "pcie" and calibration and calibration["host_curve_gbs"]
+                                         else None),
                      "peak_source": psrc,
                      "kernel_ms": kern_all[slow],
                      "how": "algorithmic bytes of the kernel's bounding term on the rank with the longest "
