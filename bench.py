@@ -219,12 +219,12 @@ def measured_peaks():
 
 
 def pcie_h2d_peak(torch) -> float:
-    """Live PCIe reference: pinned-host -> device cudaMemcpy of 1 GiB, best of 5 (GB/s)."""
+    """Live PCIe reference: pinned-host -> device cudaMemcpy of 1 GiB, best of 10 (GB/s)."""
     n = 1 << 30
     h = torch.empty(n, dtype=torch.uint8).pin_memory()
     d = torch.empty(n, dtype=torch.uint8, device="cuda")
     best = 1e9
-    for _ in range(5):
+    for _ in range(10):
         s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         s.record()
         d.copy_(h, non_blocking=True)
@@ -490,6 +490,11 @@ def main():
         del calibration["host_curve"], calibration["peer_curve"]
         log(f"calibration in {time.time() - t0:.2f}s: host_sms {cal['host_sms']} "
             f"({cal['bw_host'] / 1e9:.1f} GB/s), peer_sms {cal['peer_sms']}")
+        if ws > 1 and cal["peer_sms"] > 0 and not args.peer_sms:
+            # SMs per peer = the tolerance measured under all-to-all
+            # load; the SMs left over start on local work (host SMs stay the workload value)
+            cache.set_dedication(0, int(ugdist.max_over_ranks(float(cal["peer_sms"]))))
+            calibration["applied_peer_sms"] = True
     if args.mode == "random":
         cache.set_mode("random")
     cache.set_stream(args.stream)
@@ -709,7 +714,7 @@ def main():
     kbytes = kr["kernel_bytes"][bound]
     peak = {"hbm": hbm, "pcie": pcie_all[slow], "nvlink_in": nvl, "nvlink_out": nvl}[bound]
     psrc = {"hbm": hbm_src,
-            "pcie": "live cudaMemcpy pinned H2D 1 GiB best-of-5 on every rank at once, this run",
+            "pcie": "live cudaMemcpy pinned H2D 1 GiB best-of-10 on every rank at once, this run",
             "nvlink_in": "B200_PROFILING.md measured peer copy",
             "nvlink_out": "B200_PROFILING.md measured peer copy"}[bound]
     gat_s = kern_all[slow] / 1e3

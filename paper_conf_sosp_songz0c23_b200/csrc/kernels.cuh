@@ -102,6 +102,8 @@ struct LocateParams {
   uint32_t row_bytes;
   int32_t num_src;
   // host pre-ordering: histogram of the host rows' key ranges, built while locating
+  int32_t items;             // keys per thread per tile (1..kLocateItems): the fused kernel
+                             // sizes tiles so the batch spreads over every CTA
   int32_t hist;              // 1 = count every host entry into range_count
   uint32_t range_shift;      // range = row >> range_shift
   uint32_t *range_count;     // kMaxRanges counters, zero between launches
@@ -326,20 +328,21 @@ __device__ __forceinline__ void locate_tile(const LocateParams &p, uint64_t tile
   if (tid < kMaxSrc) s_cnt[tid] = 0;
   __syncthreads();
   const KeyT *keys = static_cast<const KeyT *>(p.keys);
-  const uint64_t tile0 = tile * (uint64_t)(THREADS * kLocateItems);
+  const int items = p.items;
+  const uint64_t tile0 = tile * (uint64_t)(THREADS * items);
 
   KeyT k[kLocateItems];
   uint64_t e[kLocateItems];
 #pragma unroll
   for (int it = 0; it < kLocateItems; ++it) {  // coalesced key loads
     const uint64_t i = tile0 + (uint64_t)it * THREADS + tid;
-    k[it] = (i < p.n) ? keys[i] : (KeyT)0;
+    k[it] = (it < items && i < p.n) ? keys[i] : (KeyT)0;
   }
 #pragma unroll
   for (int it = 0; it < kLocateItems; ++it) {  // random location-table reads, all in flight
     const uint64_t i = tile0 + (uint64_t)it * THREADS + tid;
-    e[it] = (i < p.n && key_in_range<KeyT>(k[it], p.num_rows)) ? ld_nc_u64(p.loc + (uint64_t)k[it])
-                                                               : ~0ull;
+    e[it] = (it < items && i < p.n && key_in_range<KeyT>(k[it], p.num_rows)) ? ld_nc_u64(p.loc + (uint64_t)k[it])
+                                                                             : ~0ull;
   }
   int src[kLocateItems];
   uint32_t pos[kLocateItems];
@@ -348,7 +351,7 @@ __device__ __forceinline__ void locate_tile(const LocateParams &p, uint64_t tile
   for (int it = 0; it < kLocateItems; ++it) {
     const uint64_t i = tile0 + (uint64_t)it * THREADS + tid;
     int s = -1;
-    if (i < p.n) {
+    if (it < items && i < p.n) {
       if (e[it] != ~0ull) {
         s = (int)(e[it] >> UGACHE_LOC_SRC_SHIFT);
       } else {
@@ -1433,7 +1436,7 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
   extern __shared__ __align__(16) uint32_t s_dyn[];
   __shared__ uint32_t s_cnt[kMaxSrc];
   __shared__ uint32_t s_base[kMaxSrc];
-  constexpr uint32_t kTile = kGatherThreads * kLocateItems;
+  const uint32_t kTile = kGatherThreads * (uint32_t)lp.items;
   const uint32_t ntiles = (lp.n + kTile - 1) / kTile;
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     gp.ctrl->t_start = globaltimer_ns();

@@ -81,6 +81,7 @@ struct ugache_ctx {
   int preorder = 1;                          // UGACHE_OPT_PREORDER (env UGACHE_PREORDER)
   int hist_smem = 1;                         // env UGACHE_HIST_SMEM (fused: per-CTA histogram)
   int host_segments = 2;                     // env UGACHE_HOST_SEGMENTS (ordered host copy)
+  int locate_spread = 1;                     // env UGACHE_LOCATE_SPREAD (fused: tile size from n)
   int fused = 2;                             // UGACHE_OPT_FUSED: 0 off, 1 on, 2 auto
   int early_walk = 0;                        // UGACHE_OPT_EARLY_WALK (env UGACHE_EARLY_WALK)
   int local_bulk = 2;                        // UGACHE_OPT_LOCAL_BULK (0 off, 1 on, 2 auto, 3)
@@ -450,6 +451,7 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_PREORDER")) ctx->preorder = atoi(e) != 0;
 
   if (const char *e = getenv("UGACHE_HIST_SMEM")) ctx->hist_smem = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_LOCATE_SPREAD")) ctx->locate_spread = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_HOST_SEGMENTS")) ctx->host_segments = std::max(1, std::min(8, atoi(e)));
   if (const char *e = getenv("UGACHE_LOCAL_BULK")) ctx->local_bulk = std::max(0, std::min(3, atoi(e)));
   if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
@@ -1237,6 +1239,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     lp.row_bytes = R;
     lp.num_src = ctx->cfg.num_gpus + 1;
     lp.hist = 0;
+    lp.items = ugk::kLocateItems;
     lp.range_shift = ctx->range_shift;
     lp.range_count = ctx->d_ranges;
     ugk::GatherParams gp;
@@ -1344,6 +1347,10 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
       ctx->last_fused = false;
       ctx->last_single_pass = true;
     } else if (fused) {  // K1 + K2 in one cooperative launch
+      // tiles of 512 x items keys, items the smallest count that covers the batch with one
+      // tile per CTA (up to kLocateItems): the locate work spreads over every SM
+      const uint64_t per = (n + (uint64_t)grid * ugk::kGatherThreads - 1) / ((uint64_t)grid * ugk::kGatherThreads);
+      if (ctx->locate_spread) lp.items = (int32_t)std::max<uint64_t>(1, std::min<uint64_t>(ugk::kLocateItems, per));
       if (ctx->timing) {
         UG_CUDA(ctx, cudaEventRecord(ctx->ev[0], s));
         UG_CUDA(ctx, cudaEventRecord(ctx->ev[1], s));
