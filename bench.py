@@ -464,9 +464,25 @@ def main():
             tdist.barrier()
             if rank != 0:
                 tier = synth.HostTable(max(trows, 1), wl.row_bytes, shm_path=tpath, create=False)
-    cache = UGache(table, wl.num_rows, wl.row_bytes, C, num_gpus=ws, rank=rank, device=local,
-                   policy=args.policy, plan=plan, order=order, host_sms=args.host_sms,
-                   peer_sms=args.peer_sms, host_tier=tier)
+    from paper_conf_sosp_songz0c23_b200._abi import UGACHE_ENOMEM, UGacheError
+    try:
+        cache = UGache(table, wl.num_rows, wl.row_bytes, C, num_gpus=ws, rank=rank, device=local,
+                       policy=args.policy, plan=plan, order=order, host_sms=args.host_sms,
+                       peer_sms=args.peer_sms, host_tier=tier)
+        ok = 1.0
+    except UGacheError as e:
+        if e.status != UGACHE_ENOMEM or tier is False:
+            raise
+        log(f"init with the host tier failed ({e}); every rank retries without it")
+        ok = 0.0
+    if ugdist.sum_over_ranks(ok) < ws:   # all ranks run the same configuration
+        if ok:
+            cache.close()
+        args.host_tier = False
+        tier = False
+        cache = UGache(table, wl.num_rows, wl.row_bytes, C, num_gpus=ws, rank=rank, device=local,
+                       policy=args.policy, plan=plan, order=order, host_sms=args.host_sms,
+                       peer_sms=args.peer_sms, host_tier=False)
     log(f"init (register host table, location table, slab) in {time.time() - t0:.1f}s")
     ugdist.connect(cache, order=order)
     del order

@@ -965,3 +965,34 @@ def test_cuda_graph_capture_and_replay(torch_cuda, stream_mode):
         ref, _ = oracle.gather(t.ptr, wl.num_rows, wl.row_bytes, kb)
         assert np.array_equal(out.cpu().numpy(), ref), b
     c.close()
+
+
+@pytest.mark.slow
+def test_full_size_gnn_pa_sampled_parity(torch_cuda):
+    """BASELINE configs[1] at full size in the benched launch configuration (111M x 512 B
+    rows, 500K unique Zipf(1.2) keys, c = 10 %, host tier, auto path = the fused kernel):
+    per-source counts equal the oracle's over the whole batch, and 8,192 sampled output rows
+    (plus the first and last) equal the oracle's gather of the same keys byte for byte."""
+    wl = synth.get_workload("gnn_pa")
+    N, R = wl.num_rows, wl.row_bytes
+    table = synth.HostTable(N, R)
+    table.fill()
+    from paper_conf_sosp_songz0c23_b200 import UGache
+    c = UGache(table, N, R, wl.capacity_rows, hotness=synth.hotness(wl), host_tier=True)
+    c.fill()
+    keys_np = synth.make_batch(wl, 0, 0)
+    keys = torch_cuda.from_numpy(keys_np).cuda()
+    out = c.extract(keys)
+    torch_cuda.cuda.synchronize()
+    assert c.last_extract_path() == "fused"
+    per, bad = c.last_batch_stats()
+    loc, _ = c.export_placement()
+    ref_cnt, ref_bad = source_counts(loc, keys_np, N, 1)
+    del loc
+    assert bad == ref_bad == 0 and np.array_equal(per, ref_cnt) and per[1] > 50_000
+    idx = np.concatenate([[0, len(keys_np) - 1], np.random.default_rng(91).choice(len(keys_np), 8192, replace=False)])
+    ref, _ = oracle.gather(table.ptr, N, R, keys_np[idx])
+    got = out[torch_cuda.from_numpy(idx).cuda()].cpu().numpy()
+    assert np.array_equal(got, ref)
+    c.close()
+    table.close()
