@@ -333,10 +333,11 @@ ugache_status ugache_set_dedication(ugache_ctx *ctx, int32_t host_sms, int32_t p
 ugache_status ugache_set_mode(ugache_ctx *ctx, int32_t mode);
 
 /* Tuning options (ugache_set_option); none changes the output bytes.
- *  UGACHE_OPT_HOST_ORDERING (default 1): the host CTAs of the factored gather first order
- *    the host bucket by key range so the rows in flight cover a small window of host
- *    address space (translation reach of the host aperture), then copy
- *    in that order; 0 = copy in bucket order.
+ *  UGACHE_OPT_HOST_ORDERING (default 1): a dense host bucket is ordered by key range before
+ *    it is copied (by every CTA right after the locate pass with UGACHE_OPT_PREORDER, else by
+ *    the host CTAs), so the rows in flight cover a small window of host address space
+ *    (translation reach of the host aperture); the host SMs then copy
+ *    it as two concurrent segments (env UGACHE_HOST_SEGMENTS); 0 = copy in bucket order.
  *  UGACHE_OPT_STAGE_HOST_IO (default 0): 1 = stage pinned host keys/out through device
  *    buffers + cudaMemcpyAsync instead of zero-copy access from the kernels.
  *  UGACHE_OPT_HOST_WARPS (default 12, 1..16): warps per host CTA that read host rows; the
@@ -380,10 +381,11 @@ typedef enum {
  *   Rows move through per-lane TMA shared-memory slots (cp.async.bulk in and out, up to
  *   12 KB in flight per warp).  No grid barrier and no bucket round trip for local rows.
  *   0 = off (locate | grid barrier | factored gather); 1 = always; 2 (default) = for rows of
- *   at most 1 KB and no queued peer source (G = 1, or UGACHE_INLINE_PEERS), unless the last
- *   launch on this ctx had a host bucket dense enough for
- *   range-ordered reads (scaled to this batch's size; the kernel mirrors its counts to
- *   pinned host memory, so the choice needs no synchronisation).  Ignored with
+ *   at most 1 KB and no queued peer source (G = 1, or UGACHE_INLINE_PEERS), unless this
+ *   batch is expected to have a host bucket dense enough for range-ordered reads: expected
+ *   host keys = the last launch's host count scaled to this batch's size (the kernel mirrors
+ *   its counts to pinned host memory, so the choice needs no synchronisation), or, before
+ *   the first launch of the ctx, n x plan.host_mass_frac.  Ignored with
  *   UGACHE_DEDICATE_WARPS and on the message path.  Timing reports the whole launch as
  *   the gather phase (locate = 0).
  * UGACHE_OPT_INLINE: bit mask of the sources whose rows the locating warp copies itself in
