@@ -40,15 +40,21 @@ ugache_status resolve_params(const ugache_config *cfg, int device_sms, Params *p
   if (cfg->host_sms < 0 || cfg->peer_sms < 0 || cfg->num_sms < 0) return UGACHE_EINVAL;
   const int S = cfg->num_sms ? cfg->num_sms : (device_sms > 0 ? device_sms : kDefaultNumSms);
   const int host_sms = cfg->host_sms ? cfg->host_sms : std::min(kDefaultHostSms, S - 1);
-  int peer_sms = 0;
-  if (G > 1) peer_sms = cfg->peer_sms ? cfg->peer_sms : (S - host_sms) / (G - 1);
-  if (host_sms < 1 || host_sms >= S) return UGACHE_EINVAL;
-  if (G > 1 && (peer_sms < 1 || (int64_t)host_sms + (int64_t)(G - 1) * peer_sms > S))
-    return UGACHE_EINVAL;
   const double R = (double)cfg->row_bytes;
   const double bl = cfg->bw_local > 0 ? cfg->bw_local : kDefaultBwLocal;
   const double bp = cfg->bw_peer > 0 ? cfg->bw_peer : kDefaultBwPeer;
   const double bh = cfg->bw_host > 0 ? cfg->bw_host : kDefaultBwHost;
+  int peer_sms = 0;
+  if (G > 1 && cfg->peer_sms) {
+    peer_sms = cfg->peer_sms;
+  } else if (G > 1) {
+    const int even = (S - host_sms) / (G - 1);  // the paper's split
+    const double cap = std::ceil(2.0 * (bp / (double)(G - 1)) * kPeerLatency / (kPeerRowsInFlightPerSm * R));
+    peer_sms = std::max(1, std::min(even, std::max(2, (int)cap)));
+  }
+  if (host_sms < 1 || host_sms >= S) return UGACHE_EINVAL;
+  if (G > 1 && (peer_sms < 1 || (int64_t)host_sms + (int64_t)(G - 1) * peer_sms > S))
+    return UGACHE_EINVAL;
   p->S = S;
   p->host_sms = host_sms;
   p->peer_sms = peer_sms;

@@ -19,8 +19,11 @@ B200 = dict(bw_local=6457.7e9, bw_peer=770e9, bw_host=34.4e9)
 
 
 def _plat(G, host_sms=8):
-    peer = (148 - host_sms) // max(G - 1, 1) if G > 1 else 0
-    return Platform(G=G, row_bytes=512, host_sms=host_sms, peer_sms=peer, **B200)
+    """The platform of make_config(..., host_sms=host_sms) with the library's default SMs per
+    peer (R14), so oracle and product evaluate the same model."""
+    plan, _ = solve(make_config(1000, 512, 100, num_gpus=G, host_sms=host_sms, bw_host=34.4e9), None,
+                    want_order=False)
+    return Platform(G=G, row_bytes=512, host_sms=host_sms, peer_sms=int(plan.peer_sms), **B200)
 
 
 @pytest.mark.parametrize("E,G", [(1000, 4), (20_000, 8), (50, 2)])
