@@ -83,9 +83,9 @@ typedef struct {
   double bw_peer;         /* bytes/s of NVLink ingress per GPU; 0 = default               */
   double bw_host;         /* bytes/s of host->GPU zero-copy reads; 0 = default            */
   int32_t host_sms;       /* SMs dedicated to host extraction; 0 = default  */
-  int32_t peer_sms;       /* SMs dedicated to each peer; 0 = min(floor((S-host)/(G-1))
-                             (P:1223-1225), the SMs that keep 1/(G-1) of bw_peer in flight
-                             twice over at the peer latency -- DESIGN.md R14)                 */
+  int32_t peer_sms;       /* SMs dedicated to each peer; 0 = floor((S-host)/(G-1));
+                             a measured cap (ugache_calibrate) is applied with
+                             ugache_set_dedication -- DESIGN.md R14                           */
   int32_t num_sms;        /* S; 0 = the device's SM count (148 on B200)                   */
   int32_t flags;          /* UGACHE_FLAG_* bits; other bits must be 0                     */
 } ugache_config;

@@ -175,6 +175,8 @@ struct GatherParams {
                                    // memory before the global atomics
   int32_t host_segments;           // ordered host copy: the ordered bucket is split into this many
                                    // segments read concurrently (1 = one cursor, in order)
+  int32_t local_pace;              // dense host bucket: ns a local-copy warp sleeps after each
+                                   // chunk (spreads the local burst over the host-bound step)
 };
 
 struct RandomParams {
@@ -881,6 +883,7 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
       for (uint32_t e0 = c0; e0 < c1; e0 += kRowsInFlight)
         copy_rows<kRowsInFlight>(base, p.out, R, b + e0, (int)min((uint32_t)kRowsInFlight, c1 - e0),
                                  lane);
+      if (host_dense && p.local_pace > 0) __nanosleep((unsigned)p.local_pace);
     }
   }
   finish_launch(p.ctrl, p.num_src, p.n_keys, 0);

@@ -44,14 +44,12 @@ ugache_status resolve_params(const ugache_config *cfg, int device_sms, Params *p
   const double bl = cfg->bw_local > 0 ? cfg->bw_local : kDefaultBwLocal;
   const double bp = cfg->bw_peer > 0 ? cfg->bw_peer : kDefaultBwPeer;
   const double bh = cfg->bw_host > 0 ? cfg->bw_host : kDefaultBwHost;
+  // SMs per peer: the paper's even split of the SMs left after the host.  The
+  // B200 refinement -- cap it at the NVLink tolerance -- is a
+  // measurement: ugache_calibrate under all-to-all load, applied by the caller
+  // (ugache_set_dedication; bench.py does at N > 1).  DESIGN.md R14.
   int peer_sms = 0;
-  if (G > 1 && cfg->peer_sms) {
-    peer_sms = cfg->peer_sms;
-  } else if (G > 1) {
-    const int even = (S - host_sms) / (G - 1);  // the paper's split
-    const double cap = std::ceil(2.0 * (bp / (double)(G - 1)) * kPeerLatency / (kPeerRowsInFlightPerSm * R));
-    peer_sms = std::max(1, std::min(even, std::max(2, (int)cap)));
-  }
+  if (G > 1) peer_sms = cfg->peer_sms ? cfg->peer_sms : (S - host_sms) / (G - 1);
   if (host_sms < 1 || host_sms >= S) return UGACHE_EINVAL;
   if (G > 1 && (peer_sms < 1 || (int64_t)host_sms + (int64_t)(G - 1) * peer_sms > S))
     return UGACHE_EINVAL;

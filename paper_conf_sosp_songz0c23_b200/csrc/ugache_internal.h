@@ -20,13 +20,6 @@ constexpr int kDefaultHostSms = 12;
 //  host  = calibrated zero-copy throughput of random 512-B host rows with range-ordered
 //          reads on the B200 box (tools/calibrate.py, gnn_pa: 34.4 GB/s; the sequential
 //          pinned-H2D DMA peak is 55.6 GB/s).
-// Default SMs per peer (B200 refinement of P:1223-1225, DESIGN.md
-// R14): enough SMs to keep 1/(G-1) of the NVLink ingress in flight twice over at the peer
-// load latency -- peer LDG to remote DRAM 2,036 cycles at 1.965 GHz (B300_MICROARCH.md,
-// NV18 as on B200) -- with kPeerRowsInFlightPerSm rows in flight per SM (16 warps x 8 rows,
-// the gather kernels' register path); never more than the paper's even split.
-constexpr double kPeerLatency = 1.04e-6;
-constexpr double kPeerRowsInFlightPerSm = 16 * 8;
 constexpr double kDefaultBwLocal = 6457.7e9;
 constexpr double kDefaultBwPeer = 770e9;
 constexpr double kDefaultBwHost = 34.4e9;
