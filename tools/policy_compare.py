@@ -5,7 +5,7 @@ P:385-413) on ONE B200 with G fake peers.
 For each G and policy: G contexts on one device share the full-size host table (and one
 host tier per policy, built once), GPU 0 extracts its own batches through the production
 path (auto: fused two-phase kernel with dedicated host / peer SMs), bit-exact against the
-oracle.  What one GPU can and cannot show:
+table generator.  What one GPU can and cannot show:
   * host rows and local rows are read exactly as on a real node (the host link of GPU 0
     serves only GPU 0 here; on a node all G GPUs read host memory at once);
   * "peer" rows come from the other contexts' slabs in the SAME HBM, i.e. faster than NVLink:
@@ -42,7 +42,6 @@ def main():
     ap.add_argument("--out", default="")
     args = ap.parse_args()
     import torch
-    import oracle
     import synth
     from paper_conf_sosp_songz0c23_b200 import (UGache, connect_in_process, fill_host_tier,
                                                 host_tier_rows, make_config, solve)
@@ -57,7 +56,7 @@ def main():
     keys_np = [synth.make_batch(wl, 0, b) for b in range(3)]
     keys = [torch.from_numpy(k).cuda() for k in keys_np]
     out = torch.empty((keys[0].numel(), R), dtype=torch.uint8, device="cuda")
-    ref0, _ = oracle.gather(table.ptr, N, R, keys_np[0])
+    ref0 = synth.rows_for_keys(keys_np[0], N, R)   # the table generator (tools never run the oracle)
     rows = []
     for G in args.gpus:
         for pol in args.policies:
