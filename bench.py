@@ -10,12 +10,14 @@ A step is one ugache_extract of one batch (locate + bucket + factored gather, SU
 111M x 128 fp32 rows = 56.8 GB host table, 500K unique Zipf(1.2) keys per GPU per batch,
 10 % per-GPU cache).  Prints ONE JSON line on rank 0.
 
-Timing: W warm-up steps; then K steps, each bracketed by CUDA events on the extract stream
-with a 256 MiB L2-flush write between steps (outside the events); barrier + synchronize
-on both sides; per-rank time = sum of the K event intervals; value = bytes of all ranks /
-max over ranks.  e2e: the same metric through UGache.extract with pinned HOST key and
-output buffers (H2D + extract + D2H inside the events).  --impl reference times the CPU
-oracle (oracle/gather.c) on the same batches.
+Timing: W warm-up steps; then K steps back to back on the extract stream (steady state: no
+L2 flush -- every step's rows, outputs and location-table lines exceed the 126 MB L2 and the
+steps cycle through --batches distinct key sets -- and no per-step host sync), CUDA events
+between consecutive steps; barrier + synchronize on both sides; per-rank time = sum of the K
+event intervals; value = bytes of all ranks / max over ranks.  `cold_l2`: the same K steps
+with a 256 MiB L2-flush write (and a ~50 us spin) before each, outside the events.  e2e: the
+same metric through UGache.extract with pinned HOST keys (read in place) and a stats
+readback, host wall clock.  --impl reference times the CPU oracle (oracle/gather.c).
 """
 from __future__ import annotations
 
@@ -92,7 +94,7 @@ def parse():
                     help="single pass: sources copied by the locating warps (UGACHE_OPT_INLINE)")
     ap.add_argument("--host-sms", type=int, default=0)
     ap.add_argument("--peer-sms", type=int, default=0)
-    ap.add_argument("--batches", type=int, default=4, help="distinct batches cycled per rank")
+    ap.add_argument("--batches", type=int, default=8, help="distinct batches cycled per rank")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -308,9 +310,13 @@ def setup_table(wl, rank, ws, torch_dist, alias_gb=0.0):
 
 
 def make_batches(wl, rank, nb):
+    """nb distinct seeded batches of this rank (generated in parallel host threads)."""
     import synth
+    from concurrent.futures import ThreadPoolExecutor
     t0 = time.time()
-    b = [synth.make_batch(wl, rank, i) for i in range(nb)]
+    synth.zipf_cdf(wl.table_rows[0], wl.alpha)      # build the shared CDF once
+    with ThreadPoolExecutor(max_workers=min(nb, max(1, (os.cpu_count() or 8) // 2))) as ex:
+        b = list(ex.map(lambda i: synth.make_batch(wl, rank, i), range(nb)))
     log(f"{nb} batches of {len(b[0])} keys in {time.time() - t0:.1f}s")
     return b
 
@@ -369,10 +375,11 @@ def config_dict(args, wl, ws):
                            f"{wl.table_bytes / 1e9:.0f} GB span" if getattr(args, "alias_gb", 0) and
                            wl.table_bytes > args.alias_gb * 1e9 else "full"),
             "parallelism": f"dp{ws}",
-            "l2": "256 MiB L2-flush write between timed steps (outside the events); per-step "
-                  "output > L2",
-            "launch_gap": "a ~50 us device spin precedes each timed step (outside the events) so "
-                          "the host has enqueued the step before its start event fires"}
+            "l2": "inputs larger than L2: no flush between the back-to-back timed steps; every step "
+                  "reads and writes its batch's rows (> 0.25 GB) and touches one location-table line "
+                  "per key, against a 126 MB L2, and the steps cycle through distinct key sets "
+                  "(--batches); the cold-L2 variant (256 MiB flush before each step) is cold_l2",
+            "batches": getattr(args, "batches", None)}
 
 
 def main():
@@ -515,12 +522,24 @@ def main():
     cache.set_stream(args.stream)
     cache.set_inline(host=args.inline != "none", peers=args.inline == "all")
 
-    batches = make_batches(wl, rank, max(1, min(args.batches, args.steps + args.warmup)))
+    # Distinct batches, used in order by every loop below (a cursor cycles over them): a
+    # batch comes back only after >= --batches other extracts, so no step reuses a recent
+    # batch's host rows or their address translations (on this box a host row read again
+    # within ~8 batches is served much faster -- DESIGN.md section 7).
+    nbat = max(1, args.batches, args.warmup + args.steps)
+    batches = make_batches(wl, rank, nbat)
     n = len(batches[0])
     R = wl.row_bytes
     dkeys = [torch.from_numpy(b).to(dev) for b in batches]
     out = torch.empty((n, R), dtype=torch.uint8, device=dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    cursor = [0]
+
+    def next_batch():
+        j = cursor[0] % len(dkeys)
+        cursor[0] += 1
+        return j
+
     def step(i, timed):
         with torch.cuda.stream(stream):
             flush.fill_(i & 0xFF)  # evict L2 between steps (outside the events)
@@ -531,64 +550,80 @@ def main():
         if timed:
             s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             s.record(stream)
-        cache.extract(dkeys[i % len(dkeys)], out, stream)
+        cache.extract(dkeys[i], out, stream)
         if timed:
             e.record(stream)
             return s, e
         return None
 
+    # ---- warm-up: W steps back to back --------------------------------------------------
     for i in range(args.warmup):
-        step(i, False)
+        cache.extract(dkeys[next_batch()], out, stream)
     stream.synchronize()
     ugdist.barrier()
     torch.cuda.synchronize()
     clocks = Clocks(local) if (rank == 0 and not args.no_clocks) else None  # every GPU of the node
     time.sleep(0.3 if clocks else 0)
-    evs, loc_ms, gat_ms, per_src, paths = [], [], [], [], []
+
+    # ---- timed region (the line's value): K steps back to back --------------------------
+    # Steady state, as an application streams batches: no L2 flush between steps -- every
+    # step touches far more than the 126 MB L2 (the batch's rows read and written, its
+    # location-table lines), and every step extracts a batch no recent step used -- and
+    # no per-step host synchronisation; CUDA events between consecutive steps time each step
+    # on the device.  The cold-L2 variant (256 MiB flush before every step) is `cold_l2`.
+    cache.enable_timing(False)
+    evs, paths = [], []
     launches = 0
-    cache.enable_timing(False)  # the timed steps carry no library events inside them
+    prev = torch.cuda.Event(enable_timing=True)
+    prev.record(stream)
     for i in range(args.steps):
-        evs.append(step(args.warmup + i, True))
-        per, _ = cache.last_batch_stats()  # syncs this step (after its end event)
-        per_src.append(per)
+        cache.extract(dkeys[next_batch()], out, stream)
+        e = torch.cuda.Event(enable_timing=True)
+        e.record(stream)
+        evs.append((prev, e))
+        prev = e
         launches += cache.last_launch_count()
         paths.append(cache.last_extract_path())
     stream.synchronize()
     torch.cuda.synchronize()
     ugdist.barrier()
     clk = clocks.stop() if clocks else None
-    # kernel pass: the same steps again with the library's own events around its launches
-    # (and the fused kernel's %globaltimer phase split) for the per-kernel roofline
+    step_ms = [a.elapsed_time(b) for a, b in evs]
+    # a multi-GPU step lasts as long as its slowest rank: per-step max over ranks
+    step_max = ugdist.gather_rows(step_ms).max(axis=0)
+    max_total_s = ugdist.max_over_ranks(sum(step_ms) / 1e3)
+    bytes_all = ugdist.sum_over_ranks(float(args.steps * n * R))
+    value = bytes_all / max_total_s / 1e9
+
+    # kernel pass (steady state too: no flush): the library's own events around its launch
+    # and the fused kernel's %globaltimer phase split, for the per-kernel roofline
+    loc_ms, gat_ms, phases = [], [], []
     cache.enable_timing(True)
-    phases = []
     for i in range(args.steps):
-        step(args.warmup + i, False)
+        cache.extract(dkeys[next_batch()], out, stream)
         a, b = cache.last_batch_timing()
         loc_ms.append(a)
         gat_ms.append(b)
         if cache.last_extract_path() == "fused":
             phases.append(cache.last_batch_phases())
     stream.synchronize()
-    log("per-step gather ms: " + " ".join(f"{x:.3f}" for x in gat_ms))
-    step_ms = [s.elapsed_time(e) for s, e in evs]
-    # a multi-GPU step lasts as long as its slowest rank: per-step max over ranks
-    step_max = ugdist.gather_rows(step_ms).max(axis=0)
-    my_total_s = sum(step_ms) / 1e3
-    max_total_s = ugdist.max_over_ranks(my_total_s)
-    bytes_all = ugdist.sum_over_ranks(float(args.steps * n * R))
-    value = bytes_all / max_total_s / 1e9
-
-    # throughput mode: the same batches back to back, no flush, no barrier,
-    # no per-step sync; device time of the whole run / batches
     cache.enable_timing(False)
+    log("per-step ms (steady state): " + " ".join(f"{x:.3f}" for x in step_ms))
+
+    # ---- cold L2: the same steps with a 256 MiB flush + ~50 us spin before each -----------
+    # (outside the events), per-source counts of every step
+    cold_ms, per_src = [], []
     ugdist.barrier()
-    tp_s, tp_e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    tp_s.record(stream)
     for i in range(args.steps):
-        cache.extract(dkeys[(args.warmup + i) % len(dkeys)], out, stream)
-    tp_e.record(stream)
-    stream.synchronize()
-    tp_ms = ugdist.max_over_ranks(tp_s.elapsed_time(tp_e) / 1e3) * 1e3 / args.steps
+        ev = step(next_batch(), True)
+        per, _ = cache.last_batch_stats()  # syncs this step (after its end event)
+        per_src.append(per)
+        cold_ms.append(ev[0].elapsed_time(ev[1]))
+    cold_max = ugdist.gather_rows(cold_ms).max(axis=0)
+    cold_total_s = ugdist.max_over_ranks(sum(cold_ms) / 1e3)
+    cold_value = bytes_all / cold_total_s / 1e9
+    log("per-step ms (cold L2): " + " ".join(f"{x:.3f}" for x in cold_ms))
+    tp_ms = float(np.mean(cold_max))
 
     # ---- host-only reference: the same kernels on just this batch's host keys ---------
     # (how close the whole step is to the time its host rows alone take on this box; the
@@ -596,14 +631,17 @@ def main():
     host_only = None
     if args.extra and args.mode == "factored":
         loc, _ = cache.export_placement()
-        b0 = batches[args.warmup % len(batches)]
-        hk = b0[(loc[b0] >> np.uint64(56)) == np.uint64(ws)]
+        hks = []
+        for _ in range(args.steps):             # the host keys of the next distinct batches
+            b = batches[next_batch()]
+            hks.append(np.ascontiguousarray(b[(loc[b] >> np.uint64(56)) == np.uint64(ws)]))
         del loc
-        if len(hk):
-            dhk = torch.from_numpy(np.ascontiguousarray(hk)).to(dev)
-            hout = torch.empty((len(hk), R), dtype=torch.uint8, device=dev)
-            hms = []
-            for i in range(args.steps + 2):
+        if all(len(h_) for h_ in hks):
+            hmax = max(len(h_) for h_ in hks)
+            hout = torch.empty((hmax, R), dtype=torch.uint8, device=dev)
+            dhks = [torch.from_numpy(h_).to(dev) for h_ in hks]
+            hms, hrows = [], 0
+            for i, dhk in enumerate(dhks):
                 with torch.cuda.stream(stream):
                     flush.fill_(i & 0xFF)
                     torch.cuda._sleep(100_000)
@@ -612,14 +650,14 @@ def main():
                 cache.extract(dhk, hout, stream)
                 he.record(stream)
                 stream.synchronize()
-                if i >= 2:
-                    hms.append(hs.elapsed_time(he))
-            host_only = {"host_keys": int(len(hk)), "ms": statistics.mean(hms),
-                         "host_gbs": len(hk) * R / (statistics.mean(hms) / 1e3) / 1e9,
+                hms.append(hs.elapsed_time(he))
+                hrows += dhk.numel()
+            host_only = {"host_keys": hrows / len(dhks), "ms": statistics.mean(hms),
+                         "host_gbs": hrows * R / (sum(hms) / 1e3) / 1e9,
                          "path": cache.last_extract_path(),
-                         "how": "extract of only the timed batch's host keys, same kernels, flush and "
-                                "spin as the timed steps"}
-            del dhk, hout
+                         "how": "extracts of only the host keys of distinct batches, same kernels, "
+                                "flush and spin as cold_l2"}
+            del dhks, hout
 
     # ---- parity on the full-size batch (every key, byte for byte) -------------------
     # Against the table generator itself (synth: row k's words are a function of k), a
@@ -647,7 +685,7 @@ def main():
 
     def e2e_run(staged):
         cache.set_stage_host_io(staged)
-        cache.extract(hkeys[0], hout, stream)  # warm-up (staging buffers)
+        cache.extract(hkeys[next_batch()], hout, stream)  # warm-up (staging buffers)
         stream.synchronize()
         ms = []
         for i in range(args.e2e_steps):
@@ -655,7 +693,7 @@ def main():
                 flush.fill_(i & 0xFF)
             s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             s.record(stream)
-            cache.extract(hkeys[i % len(hkeys)], hout, stream)
+            cache.extract(hkeys[next_batch()], hout, stream)
             e.record(stream)
             stream.synchronize()
             ms.append(s.elapsed_time(e))
@@ -681,7 +719,7 @@ def main():
             flush.fill_(i & 0xFF)
         stream.synchronize()
         t0 = time.perf_counter()
-        cache.extract(hkeys[i % len(hkeys)], out, stream)
+        cache.extract(hkeys[next_batch()], out, stream)
         per_e2e, bad_e2e = cache.last_batch_stats()
         dt = (time.perf_counter() - t0) * 1e3
         if i:
@@ -698,15 +736,29 @@ def main():
     if args.extra and args.mode == "factored":
         cache.set_mode("random")
         cache.enable_timing(False)  # same event placement as the timed factored steps
-        rms = []
-        for i in range(args.steps + 2):
-            r = step(i, True)
-            if i >= 2:
-                stream.synchronize()
-                rms.append(r[0].elapsed_time(r[1]))
+        for i in range(2):
+            cache.extract(dkeys[next_batch()], out, stream)
+        rprev = torch.cuda.Event(enable_timing=True)
+        rprev.record(stream)
+        rev = []
+        for i in range(args.steps):           # steady state, as the timed steps
+            cache.extract(dkeys[next_batch()], out, stream)
+            e = torch.cuda.Event(enable_timing=True)
+            e.record(stream)
+            rev.append((rprev, e))
+            rprev = e
+        stream.synchronize()
+        rms = [a.elapsed_time(b) for a, b in rev]
+        rcold = []
+        for i in range(args.steps):           # cold L2, as cold_l2
+            r = step(next_batch(), True)
+            stream.synchronize()
+            rcold.append(r[0].elapsed_time(r[1]))
         cache.set_mode("factored")
         ablation = {"random_dispatch_ms_per_step": statistics.mean(rms),
-                    "factored_ms_per_step": statistics.mean(step_ms)}
+                    "factored_ms_per_step": statistics.mean(step_ms),
+                    "cold_l2": {"random_dispatch_ms_per_step": statistics.mean(rcold),
+                                "factored_ms_per_step": statistics.mean(cold_ms)}}
 
     # ---- roofline --------------------------------------------------------------------
     peaks = measured_peaks()
@@ -775,7 +827,7 @@ def main():
                      "note": "source bytes scaled by the batch's unique fraction (per-source mix assumed "
                              "the same for repeats); output bytes stay n * R"}
     if host_only:
-        host_only["step_over_host_only"] = ms_per_step / host_only["ms"]
+        host_only["step_over_host_only"] = tp_ms / host_only["ms"]   # both cold L2
     line = {
         "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": ws, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
@@ -813,10 +865,12 @@ def main():
                       "step_ms": step_all.tolist(), "pcie_peak_gbs": pcie_all.tolist(),
                       "t_roof_us": [r_["t_roof_s"] * 1e6 for r_ in rl["ranks"]]} if ws > 1 else None),
         "ms_p50": float(np.percentile(step_max, 50)), "ms_p99": float(np.percentile(step_max, 99)),
-        "throughput_mode": {"ms_per_batch": tp_ms, "value": ugdist.sum_over_ranks(float(n * R)) / (tp_ms / 1e3) / 1e9,
-                            "unit": "GB/s",
-                            "how": "the timed batches back to back (no L2 flush, no barrier, no per-step "
-                                   "sync), device time / batches, max over ranks"},
+        "cold_l2": {"ms_per_step": tp_ms, "value": cold_value, "unit": "GB/s",
+                    "ms_p50": float(np.percentile(cold_max, 50)), "ms_p99": float(np.percentile(cold_max, 99)),
+                    "roofline_frac": (kr["kernel_bytes"][bound] / (tp_ms / 1e3) / 1e9) / peak if peak else None,
+                    "how": "the same K steps with a 256 MiB L2-flush write and a ~50 us device spin "
+                           "before each (outside the events), CUDA events per step, max over ranks; "
+                           "roofline_frac = the kernel's bounding-term bytes / the cold step time / peak"},
         "duplicate_aware": dup_aware,
         "host_only": host_only,
         "kernel_ms": {"locate_bucket": float(np.max(loc_all)),

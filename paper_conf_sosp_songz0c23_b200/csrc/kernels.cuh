@@ -177,6 +177,8 @@ struct GatherParams {
                                    // segments read concurrently (1 = one cursor, in order)
   int32_t local_pace;              // dense host bucket: ns a local-copy warp sleeps after each
                                    // chunk (spreads the local burst over the host-bound step)
+  int32_t local_warps;             // dense host bucket: warps per non-host SM copying local rows
+                                   // (0 = all 16)
 };
 
 struct RandomParams {
@@ -205,6 +207,11 @@ struct FillParams {
 // streamed rows do not push longer-lived lines (location-table sectors, the GMMU's cached
 // translations of the host aperture) out of L2 between batches.  Set at ctx init.
 __device__ __constant__ int c_row_evict_first;
+// 1 (default) = location-table lookups carry the L2 evict_first policy: the random 8-B
+// lookups (one >= 64-B line each) then stop displacing longer-lived L2 lines between batches
+// -- on the B200 box that keeps the host aperture's translation state warm from one batch
+// to the next (steady state)
+__device__ __constant__ int c_lt_evict_first;
 
 __device__ __forceinline__ uint64_t l2_policy_evict_first() {
   uint64_t pol;
@@ -228,6 +235,15 @@ __device__ __forceinline__ void st_cs_v4(void *p, const uint4 &v) {
   asm volatile("st.global.cs.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y),
                "r"(v.z), "r"(v.w)
                : "memory");
+}
+__device__ __forceinline__ uint64_t ld_lt_u64(const uint64_t *p) {  // location-table lookup
+  uint64_t r;
+  if (c_lt_evict_first) {
+    asm volatile("ld.global.nc.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(r) : "l"(p), "l"(l2_policy_evict_first()));
+  } else {
+    asm volatile("ld.global.nc.u64 %0, [%1];" : "=l"(r) : "l"(p));
+  }
+  return r;
 }
 __device__ __forceinline__ uint64_t ld_nc_u64(const uint64_t *p) {
   uint64_t r;
@@ -343,7 +359,7 @@ __device__ __forceinline__ void locate_tile(const LocateParams &p, uint64_t tile
 #pragma unroll
   for (int it = 0; it < kLocateItems; ++it) {  // random location-table reads, all in flight
     const uint64_t i = tile0 + (uint64_t)it * THREADS + tid;
-    e[it] = (it < items && i < p.n && key_in_range<KeyT>(k[it], p.num_rows)) ? ld_nc_u64(p.loc + (uint64_t)k[it])
+    e[it] = (it < items && i < p.n && key_in_range<KeyT>(k[it], p.num_rows)) ? ld_lt_u64(p.loc + (uint64_t)k[it])
                                                                              : ~0ull;
   }
   int src[kLocateItems];
@@ -606,7 +622,7 @@ __device__ __forceinline__ void host_walk_copy(const GatherParams &p, int warp, 
         const int64_t k = p.keys_u32 ? (int64_t)static_cast<const uint32_t *>(p.keys)[i]
                                      : static_cast<const int64_t *>(p.keys)[i];
         if (k >= 0 && (uint64_t)k < p.num_rows) {
-          const uint64_t l = ld_nc_u64(p.loc + k);
+          const uint64_t l = ld_lt_u64(p.loc + k);
           if ((int)(l >> UGACHE_LOC_SRC_SHIFT) == host_src) ent = ((l & UGACHE_LOC_ROW_MASK) << 32) | i;
         }
       }
@@ -864,7 +880,12 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
   // DESIGN.md section 6; 3 = on every CTA without a host role)
   const bool use_bulk = p.local_bulk == 1 || (p.local_bulk == 2 && !host_dense) ||
                         (p.local_bulk == 3 && !host_cta);
-  if (use_bulk) {
+  // dense host bucket: optionally only `local_warps` warps of each non-host SM copy local
+  // rows (a lower local request rate spread over the host-bound step)
+  const bool local_warp = !(host_dense && p.local_warps > 0 && !host_cta && warp >= p.local_warps);
+  if (!local_warp) {
+    // nothing: this warp leaves the local rows to the SM's first local_warps warps
+  } else if (use_bulk) {
     __shared__ __align__(8) uint64_t s_bars[kGatherWarps][kBulkMaxSlots];
     __shared__ uint32_t s_oidx[kGatherWarps][kBulkMaxSlots];
     local_bulk_copy(p, reinterpret_cast<uint8_t *>(s_dyn) + kRangeTabBytes + warp * kBulkWarpBytes,
@@ -1115,7 +1136,7 @@ __device__ __forceinline__ void stream_locs(const LocateParams &lp, const Gather
   for (int it = 0; it < kStreamK; ++it) {
     const uint32_t i = i0 + it * ck + lane;
     e[it] = (it < (int)K && (uint32_t)lane < ck && i < lp.n && key_in_range<KeyT>(k[it], lp.num_rows))
-                ? ld_nc_u64(lp.loc + (uint64_t)k[it])
+                ? ld_lt_u64(lp.loc + (uint64_t)k[it])
                 : ~0ull;
   }
 }
@@ -1377,7 +1398,7 @@ __device__ __forceinline__ void stream_body(const LocateParams &lp, const Gather
         const uint32_t i = cs[g] * (uint32_t)gp.stream_ck + lane;
         es[g] = (cs[g] < nchunks && (uint32_t)lane < (uint32_t)gp.stream_ck && i < n &&
                  key_in_range<KeyT>(ks[g], lp.num_rows))
-                    ? ld_nc_u64(lp.loc + (uint64_t)ks[g])
+                    ? ld_lt_u64(lp.loc + (uint64_t)ks[g])
                     : ~0ull;
       }
 #pragma unroll
@@ -1519,7 +1540,7 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
     if (lane < nvalid) {
       const KeyT k = keys[e0 + lane];
       if (key_in_range<KeyT>(k, p.num_rows)) {
-        const uint64_t e = ld_nc_u64(p.loc + (uint64_t)k);
+        const uint64_t e = ld_lt_u64(p.loc + (uint64_t)k);
         s = (int)(e >> UGACHE_LOC_SRC_SHIFT);
         rr = e & UGACHE_LOC_ROW_MASK;
       } else {

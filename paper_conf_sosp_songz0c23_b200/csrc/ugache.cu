@@ -83,6 +83,7 @@ struct ugache_ctx {
   int host_segments = 2;                     // env UGACHE_HOST_SEGMENTS (ordered host copy)
   int locate_spread = 1;                     // env UGACHE_LOCATE_SPREAD (fused: tile size from n)
   int local_pace = 0;                        // env UGACHE_LOCAL_PACE (ns, experiment)
+  int local_warps = 0;                       // env UGACHE_LOCAL_WARPS (dense host: warps per SM on local rows)
   int fused = 2;                             // UGACHE_OPT_FUSED: 0 off, 1 on, 2 auto
   int early_walk = 0;                        // UGACHE_OPT_EARLY_WALK (env UGACHE_EARLY_WALK)
   int local_bulk = 2;                        // UGACHE_OPT_LOCAL_BULK (0 off, 1 on, 2 auto, 3)
@@ -454,6 +455,7 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_HIST_SMEM")) ctx->hist_smem = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_LOCATE_SPREAD")) ctx->locate_spread = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_LOCAL_PACE")) ctx->local_pace = std::max(0, std::min(1000000, atoi(e)));
+  if (const char *e = getenv("UGACHE_LOCAL_WARPS")) ctx->local_warps = std::max(0, std::min(ugk::kGatherWarps, atoi(e)));
   if (const char *e = getenv("UGACHE_HOST_SEGMENTS")) ctx->host_segments = std::max(1, std::min(8, atoi(e)));
   if (const char *e = getenv("UGACHE_LOCAL_BULK")) ctx->local_bulk = std::max(0, std::min(3, atoi(e)));
   if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
@@ -463,6 +465,9 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
     int ef = 0;
     if (const char *e = getenv("UGACHE_ROW_EVICT_FIRST")) ef = atoi(e) != 0;
     UG_CUDA(ctx, cudaMemcpyToSymbol(ugk::c_row_evict_first, &ef, sizeof(ef)));
+    int lf = 1;
+    if (const char *e = getenv("UGACHE_LT_EVICT_FIRST")) lf = atoi(e) != 0;
+    UG_CUDA(ctx, cudaMemcpyToSymbol(ugk::c_lt_evict_first, &lf, sizeof(lf)));
   }
   if (const char *e = getenv("UGACHE_STREAM_GROUP"))
     ctx->stream_group = std::max(0, std::min(ugk::kStreamGroupMax, atoi(e)));
@@ -1300,6 +1305,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     gp.hist_smem = ctx->hist_smem;
     gp.host_segments = ctx->host_segments;
     gp.local_pace = ctx->local_pace;
+    gp.local_warps = ctx->local_warps;
     int grid = 0;
     build_roles(ctx, &gp, &grid);
     if (msg_local) {  // message baseline: no SM reads a peer; the peer buckets stay for msg_*

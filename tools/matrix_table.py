@@ -19,11 +19,12 @@ for f in sorted(os.listdir(d)):
     n = ps["local"] + ps["peer"] + ps["host"]
     ab = j.get("fem_ablation") or {}
     ho = j.get("host_only") or {}
-    rows.append("| {} | {} | {:.0%} | {} | {:.4f} | {:.0f} | {} {:.2f} | {:.2f} | {} | {} | {} |".format(
+    rr = r.get("random_row_peak") or {}
+    rows.append("| {} | {} | {:.0%} | {} | {:.4f} | {:.0f} | {} {:.2f} | {} | {:.2f} | {} | {} | {} |".format(
         c["workload"], c["keys_per_batch_per_gpu"], c["cache_ratio"], r.get("path"), j["ms_per_step"], j["value"],
-        r["bound"], r["frac"], j["source_mix_roofline"]["frac"], f"{ps['host'] / n:.1%}",
+        r["bound"], r["frac"], f"{rr['frac']:.2f}" if rr else "-", j["source_mix_roofline"]["frac"], f"{ps['host'] / n:.1%}",
         f"{ab['random_dispatch_ms_per_step']:.4f}" if ab else "-",
         f"{ho['ms']:.4f}" if ho else "-"))
-print("| workload | keys/batch | c | path | ms/batch | GB/s | kernel roofline | source-mix frac | host share | random dispatch ms | host keys alone ms |")
-print("|---|---|---|---|---|---|---|---|---|---|---|")
+print("| workload | keys/batch | c | path | ms/batch | GB/s | kernel roofline | vs random-row host peak | source-mix frac | host share | random dispatch ms | host keys alone ms |")
+print("|---|---|---|---|---|---|---|---|---|---|---|---|")
 print("\n".join(rows))
