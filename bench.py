@@ -574,14 +574,17 @@ def main():
     cache.enable_timing(False)
     evs, paths = [], []
     launches = 0
-    prev = torch.cuda.Event(enable_timing=True)
-    prev.record(stream)
+    marks = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
+    with torch.cuda.stream(stream):
+        # ~1 ms of device spin before the first mark (outside the timed region) lets the
+        # host queue the steps ahead of the device, so small batches are not timed at the
+        # Python enqueue rate
+        torch.cuda._sleep(2_000_000)
+    marks[0].record(stream)
     for i in range(args.steps):
         cache.extract(dkeys[next_batch()], out, stream)
-        e = torch.cuda.Event(enable_timing=True)
-        e.record(stream)
-        evs.append((prev, e))
-        prev = e
+        marks[i + 1].record(stream)
+        evs.append((marks[i], marks[i + 1]))
         launches += cache.last_launch_count()
         paths.append(cache.last_extract_path())
     stream.synchronize()
@@ -738,15 +741,15 @@ def main():
         cache.enable_timing(False)  # same event placement as the timed factored steps
         for i in range(2):
             cache.extract(dkeys[next_batch()], out, stream)
-        rprev = torch.cuda.Event(enable_timing=True)
-        rprev.record(stream)
+        rmarks = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
+        with torch.cuda.stream(stream):
+            torch.cuda._sleep(2_000_000)
+        rmarks[0].record(stream)
         rev = []
         for i in range(args.steps):           # steady state, as the timed steps
             cache.extract(dkeys[next_batch()], out, stream)
-            e = torch.cuda.Event(enable_timing=True)
-            e.record(stream)
-            rev.append((rprev, e))
-            rprev = e
+            rmarks[i + 1].record(stream)
+            rev.append((rmarks[i], rmarks[i + 1]))
         stream.synchronize()
         rms = [a.elapsed_time(b) for a, b in rev]
         rcold = []

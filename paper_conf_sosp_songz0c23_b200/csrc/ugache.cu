@@ -84,6 +84,8 @@ struct ugache_ctx {
   int locate_spread = 1;                     // env UGACHE_LOCATE_SPREAD (fused: tile size from n)
   int local_pace = 0;                        // env UGACHE_LOCAL_PACE (ns, experiment)
   int local_warps = 0;                       // env UGACHE_LOCAL_WARPS (dense host: warps per SM on local rows)
+  int stream_ck = 0;                         // env UGACHE_STREAM_CK (single pass: max keys per chunk)
+  int sparse_host_regpath = 1;               // env UGACHE_SPARSE_HOST_REGPATH
   int fused = 2;                             // UGACHE_OPT_FUSED: 0 off, 1 on, 2 auto
   int early_walk = 0;                        // UGACHE_OPT_EARLY_WALK (env UGACHE_EARLY_WALK)
   int local_bulk = 2;                        // UGACHE_OPT_LOCAL_BULK (0 off, 1 on, 2 auto, 3)
@@ -456,6 +458,12 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_LOCATE_SPREAD")) ctx->locate_spread = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_LOCAL_PACE")) ctx->local_pace = std::max(0, std::min(1000000, atoi(e)));
   if (const char *e = getenv("UGACHE_LOCAL_WARPS")) ctx->local_warps = std::max(0, std::min(ugk::kGatherWarps, atoi(e)));
+  if (const char *e = getenv("UGACHE_SPARSE_HOST_REGPATH")) ctx->sparse_host_regpath = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_STREAM_CK")) {
+    int v = atoi(e), ck = 4;
+    while (ck < v && ck < 32) ck <<= 1;
+    ctx->stream_ck = v > 0 ? ck : 0;
+  }
   if (const char *e = getenv("UGACHE_HOST_SEGMENTS")) ctx->host_segments = std::max(1, std::min(8, atoi(e)));
   if (const char *e = getenv("UGACHE_LOCAL_BULK")) ctx->local_bulk = std::max(0, std::min(3, atoi(e)));
   if (const char *e = getenv("UGACHE_STAGE_HOST_IO")) ctx->stage_host_io = atoi(e) != 0;
@@ -1294,6 +1302,10 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
         gp.stream_ck = (int32_t)ck;
         gp.stream_k = 1;
       }
+      if (ctx->stream_ck > 0) {  // env UGACHE_STREAM_CK: keys per chunk (4..32, power of 2)
+        gp.stream_ck = std::min<int32_t>(gp.stream_ck, ctx->stream_ck);
+        gp.stream_k = 1;
+      }
     }
     gp.stream_host_last = ctx->stream_host_last;
     gp.stream_host_cap = ctx->stream_host_cap;
@@ -1317,14 +1329,14 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     // memory by the kernel) had a host bucket dense enough for range-ordered reads; rows
     // above 1 KB stay on the two-phase path (measured faster there)
     bool stream = !msg_local && !ctx->warp_dedication && ctx->stream != 0;
+    // Expected host keys of this batch: scaled from the previous launch on this ctx (its
+    // counts mirrored to pinned host memory by the kernel, no synchronisation), or, before
+    // the first launch, from the plan's host hotness mass (keys x host_mass_frac).
+    const volatile uint32_t *m = ctx->h_mirror;
+    const uint64_t pn = m[0], ph = m[1];
+    const double exp_host = (m[2] && pn) ? (double)ph * (double)n / (double)pn
+                                         : (double)n * ctx->plan.host_mass_frac;
     if (stream && ctx->stream == 2) {
-      // Expected host keys of this batch: scaled from the previous launch on this ctx (its
-      // counts mirrored to pinned host memory by the kernel, no synchronisation), or, before
-      // the first launch, from the plan's host hotness mass (keys x host_mass_frac).
-      const volatile uint32_t *m = ctx->h_mirror;
-      const uint64_t pn = m[0], ph = m[1];
-      const double exp_host = (m[2] && pn) ? (double)ph * (double)n / (double)pn
-                                           : (double)n * ctx->plan.host_mass_frac;
       // with peer rows queued to dedicated SMs the two-phase kernel measured faster (fake
       // peers), so auto takes the single pass only without peer queues
       const bool peer_queues = ctx->cfg.num_gpus > 1 && !(ctx->inline_mask & UGACHE_INLINE_PEERS);
@@ -1332,6 +1344,14 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
                !(ctx->host_sort && exp_host >= (double)ctx->host_sort_min);
     }
     const bool fused = ctx->fused == 1 || (ctx->fused == 2 && n <= kFusedAutoMaxKeys);
+    if (stream && ctx->sparse_host_regpath && exp_host >= 0.005 * (double)n && ctx->stream_ck == 0) {
+      // a sparse but present host bucket (cold host rows, latency-bound): the register path
+      // with 16-key chunks keeps fewer host requests in flight per warp and measured faster
+      // than the TMA slots on distinct DLR-shaped batches
+      gp.stream_bulk = 0;
+      gp.stream_ck = std::min<int32_t>(gp.stream_ck, 16);
+      gp.stream_k = 1;
+    }
     if (!stream && ctx->preorder && ctx->host_sort && !gp.early_walk) {
       // two-phase paths: the locate pass builds the host range histogram, and every CTA of the
       // gather scatters a slice of the host bucket into range order (kernels.cuh preorder_host)
