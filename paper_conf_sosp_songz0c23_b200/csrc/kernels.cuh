@@ -721,6 +721,20 @@ __device__ __forceinline__ uint64_t l2_evict_first_policy() {
 __device__ __forceinline__ void bulk_wait_read_all() {
   asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
 }
+// cp.async (LDGSTS) of one 4/8-byte word into shared memory: a load with no register held
+// while it is in flight (single-pass locate pipeline, stream_prefetch = 2)
+__device__ __forceinline__ void cp_async_word(void *smem, const void *g, int bytes, bool evict_first) {
+  if (bytes == 8 && evict_first)
+    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 8, %2;" ::"r"(smem_u32(smem)), "l"(g),
+                 "l"(l2_policy_evict_first())
+                 : "memory");
+  else if (bytes == 8)
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(smem)), "l"(g) : "memory");
+  else
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(smem)), "l"(g) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 
 // Local bucket drained by TMA bulk copies (A4 on B200): each row goes HBM -> shared memory
@@ -1353,7 +1367,50 @@ __device__ __forceinline__ void stream_body(const LocateParams &lp, const Gather
     }
     return __shfl_sync(kFullMask, c, 0);
   };
-  if (my_src < 0 && gp.stream_prefetch) {
+  if (my_src < 0 && gp.stream_prefetch == 2 && gp.stream_k == 1 && gp.stream_ck == 32) {
+    // locating warp, pipelined through shared memory with cp.async (no register holds a
+    // load in flight): the keys of chunk i+2 and the location entries of chunk i+1 land
+    // while chunk i's rows are fed to the slots, so the key -> entry dependent loads leave
+    // the warp's critical path.  Each lane stages only its own key / entry (lane-private
+    // words: cp.async.wait_group alone orders them).  Entries alternate between two
+    // buffers so a new entry never lands on one that is still being read.
+    __shared__ __align__(8) uint64_t s_pf[kGatherWarps][3][32];
+    KeyT *pk = reinterpret_cast<KeyT *>(s_pf[warp][0]);
+    const KeyT *keys = static_cast<const KeyT *>(lp.keys);
+    const bool ef = c_lt_evict_first != 0;
+    auto lane_key = [&](uint32_t c) { return c < nchunks && c * 32u + (uint32_t)lane < n; };
+    uint32_t c0 = claim_chunk(), c1 = kNoClaim, buf = 0;
+    bool v0 = false;  // this lane's key of chunk c0 is in range (its entry is staged)
+    if (c0 < nchunks) {
+      if (lane_key(c0)) {
+        const KeyT k = keys[c0 * 32u + lane];
+        v0 = key_in_range<KeyT>(k, lp.num_rows);
+        if (v0) cp_async_word(&s_pf[warp][1][lane], lp.loc + (uint64_t)k, 8, ef);
+      }
+      c1 = claim_chunk();
+      if (lane_key(c1)) cp_async_word(&pk[lane], keys + c1 * 32u + lane, (int)sizeof(KeyT), false);
+    }
+    cp_async_commit();
+    while (c0 < nchunks) {
+      cp_async_wait_all();
+      uint64_t e[kStreamK];
+#pragma unroll
+      for (int it = 0; it < kStreamK; ++it) e[it] = ~0ull;
+      e[0] = v0 ? s_pf[warp][1 + buf][lane] : ~0ull;
+      const uint32_t c2 = c1 < nchunks ? claim_chunk() : kNoClaim;
+      bool v1 = false;
+      if (lane_key(c1)) {
+        const KeyT k = pk[lane];
+        v1 = key_in_range<KeyT>(k, lp.num_rows);
+        if (v1) cp_async_word(&s_pf[warp][2 - buf][lane], lp.loc + (uint64_t)k, 8, ef);
+      }
+      if (lane_key(c2)) cp_async_word(&pk[lane], keys + c2 * 32u + lane, (int)sizeof(KeyT), false);
+      cp_async_commit();
+      stream_chunk_located<KeyT>(lp, gp, c0, e, lane, s_addr, s_idx, s_inl, sl);
+      c0 = c1, c1 = c2, v0 = v1, buf ^= 1u;
+    }
+    cp_async_wait_all();
+  } else if (my_src < 0 && gp.stream_prefetch) {
     // locating warp, software-pipelined two deep: the keys of chunk i+2 and the location
     // entries of chunk i+1 are in flight while chunk i's rows are fed to the slots
     KeyT k1[kStreamK];

@@ -484,7 +484,7 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
     ctx->stream_peer_warps = std::max(1, std::min(ugk::kGatherWarps, atoi(e)));
   if (const char *e = getenv("UGACHE_STREAM_REGSTORE")) ctx->stream_regstore = atoi(e) != 0;
   if (const char *e = getenv("UGACHE_STREAM_COOP")) ctx->stream_coop = atoi(e) != 0;
-  if (const char *e = getenv("UGACHE_STREAM_PREFETCH")) ctx->stream_prefetch = atoi(e) != 0;
+  if (const char *e = getenv("UGACHE_STREAM_PREFETCH")) ctx->stream_prefetch = atoi(e);
   if (const char *e = getenv("UGACHE_STREAM_NAP")) ctx->stream_nap = std::max(0, atoi(e));
   if (const char *e = getenv("UGACHE_STREAM_STATIC")) ctx->stream_static = std::max(0, atoi(e));
   if (const char *e = getenv("UGACHE_STREAM_HOST_CAP")) ctx->stream_host_cap = std::max(0, atoi(e));

@@ -696,6 +696,31 @@ def test_single_pass_register_store_retire(torch_cuda, monkeypatch, G):
             g.close()
 
 
+@pytest.mark.parametrize("prefetch", ["1", "2"])
+@pytest.mark.parametrize("sched", ["0", "1", "2"])
+@pytest.mark.parametrize("key_dtype", [np.int64, np.uint32])
+def test_single_pass_locate_pipeline(torch_cuda, monkeypatch, prefetch, sched, key_dtype):
+    """Single pass with the locating warps pipelined (UGACHE_STREAM_PREFETCH: 1 registers,
+    2 shared memory via cp.async): every chunk's entries are the ones of its own keys, for
+    both key types, every chunk schedule, queued peers, inline host rows, out-of-range keys,
+    ragged and tiny batches."""
+    monkeypatch.setenv("UGACHE_STREAM_PREFETCH", prefetch)
+    monkeypatch.setenv("UGACHE_STREAM_STATIC", sched)
+    N, R = 200_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(57).permutation(N)]
+    for G in (1, 4):
+        t, group_ = make_group(torch_cuda, N, R, 6000, G, h)
+        c = group_[0]
+        c.set_stream("on")
+        for n in (1, 31, 33, 4_999, 150_001, 700_000):
+            keys = np.random.default_rng(n).integers(0, N + 2, n)
+            if key_dtype == np.int64:
+                keys[::97] = -5
+            check_batch(torch_cuda, c, t, keys, N, R, G, key_dtype=key_dtype)
+        for g in group_:
+            g.close()
+
+
 def test_fused_phase_stamps(torch_cuda):
     """ugache_last_batch_phases: after a fused launch with a dense host bucket the stamps are
     ordered (locate <= host ordered <= host copies done <= the launch's event time); after a
