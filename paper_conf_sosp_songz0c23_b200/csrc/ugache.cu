@@ -1257,7 +1257,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     lp.items = ugk::kLocateItems;
     lp.range_shift = ctx->range_shift;
     lp.range_count = ctx->d_ranges;
-    ugk::GatherParams gp;
+    ugk::GatherParams gp{};
     gp.buckets = ctx->d_buckets;
     gp.ctrl = ctx->d_ctrl;
     for (int j = 0; j < ugk::kMaxSrc; ++j) gp.base[j] = ctx->src_base[j];
