@@ -1325,6 +1325,12 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
       gp.peer_sms = 0;
       gp.host_sms_max = ctx->host_dynamic ? std::max(ctx->host_sms, gp.num_sms) : ctx->host_sms;
     }
+    // A sparse host bucket is walked in input order by the host-role SMs (host_walk), which
+    // re-reads every key's location entry: that pays only when most SMs walk (G = 1).  With
+    // peer roles holding most SMs the walkers are few (12-15 at G = 2..8) and the walk took
+    // 0.40-0.50 ms for 3-4K host rows of a 500K-key batch, against 0.16 ms ordered
+    // (placement grid), so there every non-empty host bucket is ordered.
+    if (ctx->host_walk && 2 * gp.host_sms_max < gp.num_sms) gp.host_sort_min = 1;
     // single pass unless the last launch on this ctx (its counts mirrored to pinned host
     // memory by the kernel) had a host bucket dense enough for range-ordered reads; rows
     // above 1 KB stay on the two-phase path (measured faster there)

@@ -721,6 +721,31 @@ def test_single_pass_locate_pipeline(torch_cuda, monkeypatch, prefetch, sched, k
             g.close()
 
 
+@pytest.mark.parametrize("G", [1, 4])
+def test_sparse_host_bucket_walk_or_order(torch_cuda, G):
+    """A sparse host bucket (far below the ordering threshold) on the two-phase kernel: with
+    G = 1 every SM walks the batch in input order (no ordering stamp); with peer roles holding
+    most SMs (G = 4) the walkers would be few, so the bucket is range-ordered instead (the
+    ordering stamp is set).  Bit-exact either way, out-of-range keys included."""
+    N, R = 300_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(58).permutation(N)]
+    C = 295_000 // G   # ~1.7 % of uniform keys on the host: < 4096 of 200K
+    t, group = make_group(torch_cuda, N, R, C, G, h, policy="partition")
+    c = group[0]
+    c.enable_timing(True)
+    c.set_stream("off")
+    rng = np.random.default_rng(59)
+    for n in (200_000, 77_777):
+        keys = rng.integers(0, N + 2, n)
+        per = check_batch(torch_cuda, c, t, keys, N, R, G)
+        assert 0 < per[G] < 4096, per
+        assert c.last_extract_path() == "fused"
+        _, ordered, _, _, _ = c.last_batch_phases()
+        assert (ordered > 0) == (G > 1), (G, ordered)
+    for g in group:
+        g.close()
+
+
 def test_fused_phase_stamps(torch_cuda):
     """ugache_last_batch_phases: after a fused launch with a dense host bucket the stamps are
     ordered (locate <= host ordered <= host copies done <= the launch's event time); after a
