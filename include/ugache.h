@@ -383,7 +383,9 @@ typedef enum {
  *   Rows move through per-lane TMA shared-memory slots (cp.async.bulk in and out, up to
  *   12 KB in flight per warp).  No grid barrier and no bucket round trip for local rows.
  *   0 = off (locate | grid barrier | factored gather); 1 = always; 2 (default) = for rows of
- *   at most 1 KB and no queued peer source (G = 1, or UGACHE_INLINE_PEERS), unless this
+ *   at most 1 KB and no queued peer source (G = 1, or UGACHE_INLINE_PEERS, or a small batch
+ *   of at most 32768 keys -- env UGACHE_SMALL_BATCH -- whose peer rows are then read inline:
+ *   a latency-bound batch saturates no link, so dedication buys nothing), unless this
  *   batch is expected to have a host bucket dense enough for range-ordered reads: expected
  *   host keys = the last launch's host count scaled to this batch's size (the kernel mirrors
  *   its counts to pinned host memory, so the choice needs no synchronisation), or, before
@@ -433,6 +435,17 @@ ugache_status ugache_last_batch_timing(ugache_ctx *ctx, float *ms_locate, float 
  * Synchronises with the last extract.  ESTATE when the last extract was not a fused
  * launch. */
 ugache_status ugache_last_batch_phases(ugache_ctx *ctx, float *ms);
+
+/* Per-CTA role timeline of the last fused (K1+K2) launch, for the paper's per-source time
+ * split (Fig. 8's picture; §5.3): one CTA per SM, listed in the chip-spreading
+ * order the roles are assigned in.  out[5*i .. 5*i+4] for position i = {role source id (GPU
+ * j = peer j or this rank = local, num_gpus = host), CTA start, gather start (grid barrier
+ * and host pre-ordering done), own role done (local padding follows), CTA done}, times in
+ * ms from the kernel's start.  out: caller-owned, 5 * (SM count) floats (<= 5 * 256);
+ * *num_ctas = SM count.  Needs ugache_enable_timing(ctx, 1) before the extract (the stamps
+ * cost four %globaltimer reads per CTA).  Synchronises with the last extract.  ESTATE when
+ * the last extract was not a fused launch with timing on. */
+ugache_status ugache_last_batch_timeline(ugache_ctx *ctx, float *out, int32_t *num_ctas);
 
 /* Number of kernel launches the last extract issued (for launch accounting). */
 ugache_status ugache_last_launch_count(const ugache_ctx *ctx, int32_t *launches);

@@ -121,6 +121,7 @@ SIGNATURES = {
     "ugache_last_launch_count": (_ST, [_P, ctypes.POINTER(_c.c_int32)]),
     "ugache_last_extract_path": (_ST, [_P, ctypes.POINTER(_c.c_int32)]),
     "ugache_last_batch_phases": (_ST, [_P, ctypes.POINTER(_c.c_float)]),
+    "ugache_last_batch_timeline": (_ST, [_P, ctypes.POINTER(_c.c_float), ctypes.POINTER(_c.c_int32)]),
     "ugache_export_placement": (_ST, [_P, _P, _P, ctypes.POINTER(_c.c_uint64)]),
     "ugache_read_slab": (_ST, [_P, _c.c_uint64, _c.c_uint64, _P]),
     "ugache_destroy": (_ST, [_P]),

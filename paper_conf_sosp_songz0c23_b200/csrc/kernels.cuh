@@ -66,7 +66,11 @@ struct Ctrl {
   unsigned long long t_loc_last;  // t_loc_max of the last launch (published by finish_launch)
   unsigned long long t_end;       // %globaltimer when the last CTA of the last launch finished
   // pinned, device-mapped host words {n, host count, launches} written by the last CTA of
-  // every launch: the host picks the next batch's path from them without synchronising
+  // every launch: the host picks the next batch's path from them without synchronising.
+  // The launch count is kept here (mirror_seq) so the kernel only WRITES host memory: a
+  // read of the mirror would put a PCIe round trip (and a cold translation) on every
+  // launch's tail.
+  uint32_t mirror_seq;
   volatile uint32_t *host_mirror;
 };
 
@@ -126,6 +130,8 @@ struct GatherParams {
   int32_t n_peers;                 // G - 1
   int32_t peer_src[kMaxSrc];       // the peer GPU ids, in role order
   uint32_t host_sort_min;          // host keys needed for range-ordered reads
+  uint32_t host_dense_min;         // host keys that make the batch PCIe-bound (the ctx's
+                                   // ordering threshold; host_sort_min may be lowered below it)
   uint8_t sm_pos[kMaxSmId];        // position of SM %smid in the chip-spreading order
   // host range ordering
   uint64_t *host_sorted;           // bucket_cap entries of scratch
@@ -179,7 +185,13 @@ struct GatherParams {
                                    // chunk (spreads the local burst over the host-bound step)
   int32_t local_warps;             // dense host bucket: warps per non-host SM copying local rows
                                    // (0 = all 16)
+  unsigned long long *timeline;    // per-CTA role timeline (timing on): kTimelineWords per
+                                   // chip position, see gather_body; nullptr = off
 };
+// Per-CTA role timeline (fused kernel, diagnostics): [role source, CTA start, gather start
+// (after the grid barrier and pre-ordering), own role done (last warp), CTA done (last
+// warp)], %globaltimer ns; zeroed by the host before each timed launch.
+constexpr int kTimelineWords = 5;
 
 struct RandomParams {
   const void *keys;
@@ -293,44 +305,59 @@ __device__ __forceinline__ bool key_in_range(KeyT k, uint64_t N) {
 }
 
 // Last CTA of a gather launch publishes stats and re-arms the control block.
+// The last CTA of a launch publishes the batch's statistics and re-arms the control block
+// for the next launch.  Its threads split the work (one source per thread, the scalar resets
+// on another warp): a single thread doing it all chained ~20 dependent L2 round trips (and,
+// before mirror_seq, a PCIe read) onto every launch's tail -- 5-7 us at G = 8.
 __device__ __forceinline__ void finish_launch(Ctrl *ctrl, int num_src, uint32_t n, uint32_t streamed) {
+  __shared__ uint32_t s_last;
   __syncthreads();
   if (threadIdx.x == 0) {
     __threadfence();
-    const uint32_t prev = atomicAdd(&ctrl->done, 1u);
-    if (prev == gridDim.x - 1) {
-      __threadfence();
-      volatile Ctrl *c = ctrl;
-      for (int s = 0; s < num_src; ++s) {
-        c->stat_counts[s] = c->counts[s];
-        c->counts[s] = 0;
-        c->qhead[s] = 0;
-      }
-      c->chunk_cursor = 0;
-      c->keys_done = 0;
-      c->stat_n = n;
-      c->last_stream = streamed;
-      if (c->host_mirror) {
-        c->host_mirror[0] = n;
-        c->host_mirror[1] = c->stat_counts[num_src - 1];
-        c->host_mirror[2] = c->host_mirror[2] + 1;
-      }
-      c->stat_bad = c->bad;
-      c->bad = 0;
-      c->local_cursor = 0;
-      c->host_arrive[0] = 0;
-      c->host_arrive[1] = 0;
-      c->host_cursor = 0;
-      for (int k = 0; k < 8; ++k) c->host_seg_cursor[k] = 0;
-      c->grid_arrive = 0;
-      c->walk_cursor = 0;
-      c->pre_arrive = 0;
-      c->t_loc_last = c->t_loc_max;
-      c->t_loc_max = 0;
-      c->t_end = globaltimer_ns();
-      __threadfence();
-      c->done = 0;
+    s_last = atomicAdd(&ctrl->done, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  volatile Ctrl *c = ctrl;
+  const int t = threadIdx.x;
+  if (t < num_src) {
+    const uint32_t v = c->counts[t];
+    c->stat_counts[t] = v;
+    c->counts[t] = 0;
+    c->qhead[t] = 0;
+    if (t == num_src - 1 && c->host_mirror) c->host_mirror[1] = v;
+  } else if (t >= 32 && t < 40) {
+    c->host_seg_cursor[t - 32] = 0;
+  } else if (t == 64) {
+    c->stat_bad = c->bad;
+    c->bad = 0;
+    c->t_loc_last = c->t_loc_max;
+    c->t_loc_max = 0;
+  } else if (t == 96) {
+    c->chunk_cursor = 0;
+    c->keys_done = 0;
+    c->stat_n = n;
+    c->last_stream = streamed;
+    c->local_cursor = 0;
+    c->host_arrive[0] = 0;
+    c->host_arrive[1] = 0;
+    c->host_cursor = 0;
+    c->grid_arrive = 0;
+    c->walk_cursor = 0;
+    c->pre_arrive = 0;
+  }
+  __syncthreads();
+  if (t == 0) {
+    if (c->host_mirror) {
+      const uint32_t seq = c->mirror_seq + 1;
+      c->mirror_seq = seq;
+      c->host_mirror[0] = n;
+      c->host_mirror[2] = seq;
     }
+    c->t_end = globaltimer_ns();
+    __threadfence();
+    c->done = 0;
   }
 }
 
@@ -737,6 +764,15 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 
+// Rows per local-cursor claim: kLocalChunk for big buckets; smaller (a multiple of 8, at
+// least 8) when the bucket would leave warps of the grid without a claim, so a medium batch
+// spreads its local rows over every warp instead of chaining 8 dependent steps on a few.
+__device__ __forceinline__ uint32_t local_chunk_rows(uint32_t cnt, int num_sms) {
+  const uint32_t warps = (uint32_t)num_sms * kGatherWarps;
+  const uint32_t per = (cnt + warps - 1) / warps;
+  return min((uint32_t)kLocalChunk, max(8u, (per + 7u) & ~7u));
+}
+
 // Local bucket drained by TMA bulk copies (A4 on B200): each row goes HBM -> shared memory
 // -> HBM as two cp.async.bulk operations, no registers hold row data, so one SM keeps
 // 16 warps x 24 rows = 196 KB in flight (LDG.128 at 128 registers/thread: 64 KB).  Lane u
@@ -772,11 +808,12 @@ __device__ __forceinline__ void local_bulk_copy(const GatherParams &p, uint8_t *
     }
   };
   uint32_t next = 0;
-  if (lane == 0) next = atomicAdd(&p.ctrl->local_cursor, (uint32_t)kLocalChunk);
+  const uint32_t lc = local_chunk_rows(cnt, p.num_sms);
+  if (lane == 0) next = atomicAdd(&p.ctrl->local_cursor, lc);
   next = __shfl_sync(kFullMask, next, 0);
   while (next < cnt) {
-    const uint32_t c0 = next, c1 = min(cnt, c0 + (uint32_t)kLocalChunk);
-    if (lane == 0) next = atomicAdd(&p.ctrl->local_cursor, (uint32_t)kLocalChunk);  // prefetch claim
+    const uint32_t c0 = next, c1 = min(cnt, c0 + lc);
+    if (lane == 0) next = atomicAdd(&p.ctrl->local_cursor, lc);  // prefetch claim
     next = __shfl_sync(kFullMask, next, 0);
     for (uint32_t e0 = c0; e0 < c1; e0 += (uint32_t)U, ++g) {
       const int d = (int)(g % (uint32_t)depth);
@@ -807,6 +844,8 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
   const int pos = smid < (uint32_t)kMaxSmId ? p.sm_pos[smid] : p.num_sms - 1;
   const int host_src = p.num_src - 1;
   if (p.preorder) preorder_host(p, s_dyn, blockIdx.x, gridDim.x);
+  unsigned long long *tl = p.timeline ? p.timeline + pos * kTimelineWords : nullptr;
+  if (tl && threadIdx.x == 0) tl[2] = globaltimer_ns();
   const uint32_t n_host = p.ctrl->counts[host_src];
   const bool host_dense = p.host_sort && n_host >= p.host_sort_min;
   const uint32_t R = p.row_bytes;
@@ -878,6 +917,10 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
                 (uint32_t)role_ctas * kGatherWarps, lane, my_src == host_src ? p.host_rows : kRowsInFlight);
 
   }
+  if (tl) {  // own role done: the CTA's last warp to leave its role (local padding follows)
+    if (threadIdx.x == 0) tl[0] = (unsigned long long)my_src;
+    if (lane == 0) atomicMax(&tl[3], globaltimer_ns());
+  }
   }
   // Dense host bucket: optionally only `local_sms` SMs (in chip-spreading order, after the
   // host / peer roles) copy local rows, spreading the local burst over the host-bound step
@@ -892,7 +935,10 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
   // TMA bulk local copies (1 always; 2 = unless the host bucket is dense -- with a
   // PCIe-bound batch the register path's gentler local burst keeps the host reads faster,
   // DESIGN.md section 6; 3 = on every CTA without a host role)
-  const bool use_bulk = p.local_bulk == 1 || (p.local_bulk == 2 && !host_dense) ||
+  // "dense" for the local path means PCIe-bound by the ctx's own threshold: a host bucket
+  // ordered only because few SMs would walk it (G > 1) is no reason to slow the local burst
+  const bool pcie_bound = host_dense && n_host >= p.host_dense_min;
+  const bool use_bulk = p.local_bulk == 1 || (p.local_bulk == 2 && !pcie_bound) ||
                         (p.local_bulk == 3 && !host_cta);
   // dense host bucket: optionally only `local_warps` warps of each non-host SM copy local
   // rows (a lower local request rate spread over the host-bound step)
@@ -909,11 +955,12 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
     const uint64_t *b = p.buckets + (uint64_t)p.local_src * p.bucket_cap;
     const uint8_t *base = p.base[p.local_src];
     uint32_t next = 0;
-    if (lane == 0) next = atomicAdd(&p.ctrl->local_cursor, (uint32_t)kLocalChunk);
+    const uint32_t lc = local_chunk_rows(cnt, p.num_sms);
+    if (lane == 0) next = atomicAdd(&p.ctrl->local_cursor, lc);
     next = __shfl_sync(kFullMask, next, 0);
     while (next < cnt) {
-      const uint32_t c0 = next, c1 = min(cnt, c0 + (uint32_t)kLocalChunk);
-      if (lane == 0) next = atomicAdd(&p.ctrl->local_cursor, (uint32_t)kLocalChunk);  // prefetch claim
+      const uint32_t c0 = next, c1 = min(cnt, c0 + lc);
+      if (lane == 0) next = atomicAdd(&p.ctrl->local_cursor, lc);  // prefetch claim
       next = __shfl_sync(kFullMask, next, 0);
       for (uint32_t e0 = c0; e0 < c1; e0 += kRowsInFlight)
         copy_rows<kRowsInFlight>(base, p.out, R, b + e0, (int)min((uint32_t)kRowsInFlight, c1 - e0),
@@ -921,6 +968,7 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
       if (host_dense && p.local_pace > 0) __nanosleep((unsigned)p.local_pace);
     }
   }
+  if (tl && lane == 0) atomicMax(&tl[4], globaltimer_ns());
   finish_launch(p.ctrl, p.num_src, p.n_keys, 0);
 }
 
@@ -1534,6 +1582,7 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
   uint32_t smid;
   asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
   const uint32_t pos = smid < (uint32_t)kMaxSmId ? gp.sm_pos[smid] : blockIdx.x;
+  if (gp.timeline && threadIdx.x == 0) gp.timeline[pos * kTimelineWords + 1] = globaltimer_ns();
   const bool walker = gp.early_walk && pos >= ntiles;
   const uint32_t arrivals = gp.early_walk ? min(gridDim.x, ntiles) : gridDim.x;
   uint32_t *s_hist = (lp.hist && gp.hist_smem) ? s_dyn : nullptr;  // the range-table area

@@ -59,6 +59,7 @@ struct ugache_ctx {
   bool filled = false;
   // scratch
   ugk::Ctrl *d_ctrl = nullptr;
+  unsigned long long *d_timeline = nullptr;  // per-CTA role timeline (kMaxSmId x kTimelineWords)
   uint64_t *d_buckets = nullptr;
   uint64_t bucket_cap = 0;
   void *d_keys_stage = nullptr;
@@ -83,6 +84,10 @@ struct ugache_ctx {
   int host_segments = 2;                     // env UGACHE_HOST_SEGMENTS (ordered host copy)
   int locate_spread = 1;                     // env UGACHE_LOCATE_SPREAD (fused: tile size from n)
   int local_pace = 0;                        // env UGACHE_LOCAL_PACE (ns, experiment)
+  uint64_t small_batch_keys = 32768;         // env UGACHE_SMALL_BATCH: auto path reads peers inline
+                                             // in the single pass up to this many keys
+  uint64_t walk_keys_per_sm = 1024;          // env UGACHE_WALK_KEYS_PER_SM: a sparse host bucket is
+                                             // walked only if keys <= walkers x this (else ordered)
   int local_warps = 0;                       // env UGACHE_LOCAL_WARPS (dense host: warps per SM on local rows)
   int stream_ck = 0;                         // env UGACHE_STREAM_CK (single pass: max keys per chunk)
   int sparse_host_regpath = 1;               // env UGACHE_SPARSE_HOST_REGPATH
@@ -300,6 +305,7 @@ void build_roles(const ugache_ctx *ctx, ugk::GatherParams *gp, int *grid) {
   gp->host_sms_max = ctx->host_dynamic ? std::max(ctx->host_sms, S - gp->n_peers * gp->peer_sms)
                                        : ctx->host_sms;
   gp->host_sort_min = ctx->host_sort_min;
+  gp->host_dense_min = ctx->host_sort_min;
   gp->warp_dedication = ctx->warp_dedication;
   gp->host_rows = ctx->host_rows;
   gp->peer_warps = ctx->wd_peer_warps;
@@ -423,6 +429,7 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   ctx->h_slot_keys.assign(slots.begin(), slots.begin() + (ptrdiff_t)ctx->n_slots);
   UG_CUDA(ctx, cudaMalloc(&ctx->d_ctrl, sizeof(ugk::Ctrl)));
   UG_CUDA(ctx, cudaMemset(ctx->d_ctrl, 0, sizeof(ugk::Ctrl)));
+  UG_CUDA(ctx, cudaMalloc(&ctx->d_timeline, ugk::kMaxSmId * ugk::kTimelineWords * sizeof(unsigned long long)));
   {  // pinned mirror of the last launch's {n, host count, launches} (path choice, K3)
     UG_CUDA(ctx, cudaHostAlloc(reinterpret_cast<void **>(&ctx->h_mirror), 4 * sizeof(uint32_t),
                                cudaHostAllocMapped));
@@ -477,6 +484,9 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
     if (const char *e = getenv("UGACHE_LT_EVICT_FIRST")) lf = atoi(e) != 0;
     UG_CUDA(ctx, cudaMemcpyToSymbol(ugk::c_lt_evict_first, &lf, sizeof(lf)));
   }
+  if (const char *e = getenv("UGACHE_INLINE")) ctx->inline_mask = atoi(e) & (UGACHE_INLINE_HOST | UGACHE_INLINE_PEERS);
+  if (const char *e = getenv("UGACHE_SMALL_BATCH")) ctx->small_batch_keys = strtoull(e, nullptr, 10);
+  if (const char *e = getenv("UGACHE_WALK_KEYS_PER_SM")) ctx->walk_keys_per_sm = strtoull(e, nullptr, 10);
   if (const char *e = getenv("UGACHE_STREAM_GROUP"))
     ctx->stream_group = std::max(0, std::min(ugk::kStreamGroupMax, atoi(e)));
   if (const char *e = getenv("UGACHE_LOCAL_SMS")) ctx->local_sms = std::max(0, atoi(e));
@@ -1318,6 +1328,9 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     gp.host_segments = ctx->host_segments;
     gp.local_pace = ctx->local_pace;
     gp.local_warps = ctx->local_warps;
+    gp.timeline = ctx->timing ? ctx->d_timeline : nullptr;
+    if (gp.timeline)
+      UG_CUDA(ctx, cudaMemsetAsync(gp.timeline, 0, ugk::kMaxSmId * ugk::kTimelineWords * sizeof(unsigned long long), s));
     int grid = 0;
     build_roles(ctx, &gp, &grid);
     if (msg_local) {  // message baseline: no SM reads a peer; the peer buckets stay for msg_*
@@ -1330,7 +1343,9 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
     // peer roles holding most SMs the walkers are few (12-15 at G = 2..8) and the walk took
     // 0.40-0.50 ms for 3-4K host rows of a 500K-key batch, against 0.16 ms ordered
     // (placement grid), so there every non-empty host bucket is ordered.
-    if (ctx->host_walk && 2 * gp.host_sms_max < gp.num_sms) gp.host_sort_min = 1;
+    if (ctx->host_walk && 2 * gp.host_sms_max < gp.num_sms &&
+        n > (uint64_t)gp.host_sms_max * ctx->walk_keys_per_sm)
+      gp.host_sort_min = 1;
     // single pass unless the last launch on this ctx (its counts mirrored to pinned host
     // memory by the kernel) had a host bucket dense enough for range-ordered reads; rows
     // above 1 KB stay on the two-phase path (measured faster there)
@@ -1346,8 +1361,17 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
       // with peer rows queued to dedicated SMs the two-phase kernel measured faster (fake
       // peers), so auto takes the single pass only without peer queues
       const bool peer_queues = ctx->cfg.num_gpus > 1 && !(ctx->inline_mask & UGACHE_INLINE_PEERS);
-      stream = R <= kStreamAutoMaxRow && !peer_queues &&
+      // A small batch is latency-bound: its rows fit in flight at once and no link saturates,
+      // so dedication buys nothing while the two-phase kernel's grid barrier puts every
+      // row's latency behind the whole locate pass; it takes the single pass with its peer
+      // rows read inline (fake peers, 2K-20K keys: 25-37 us -> 12-22 us)
+      const bool small = n <= ctx->small_batch_keys;
+      stream = R <= kStreamAutoMaxRow && (!peer_queues || small) &&
                !(ctx->host_sort && exp_host >= (double)ctx->host_sort_min);
+      if (stream && peer_queues) {
+        gp.inline_peer = 1;
+        gp.stream_queues = !gp.inline_host && ctx->host_sms > 0;
+      }
     }
     const bool fused = ctx->fused == 1 || (ctx->fused == 2 && n <= kFusedAutoMaxKeys);
     if (stream && ctx->sparse_host_regpath && exp_host >= 0.005 * (double)n && ctx->stream_ck == 0) {
@@ -1604,6 +1628,28 @@ ugache_status ugache_last_batch_phases(ugache_ctx *ctx, float *ms) {
   return UGACHE_OK;
 }
 
+ugache_status ugache_last_batch_timeline(ugache_ctx *ctx, float *out, int32_t *num_ctas) {
+  if (!ctx || !out || !num_ctas) return UGACHE_EINVAL;
+  if (!ctx->last_fused || ctx->last_launches == 0 || ctx->mode != UGACHE_MODE_FACTORED || !ctx->timing)
+    return fail(ctx, UGACHE_ESTATE, "last extract was not a fused launch with timing on");
+  ugache_status st = begin(ctx);
+  if (st != UGACHE_OK) return st;
+  UG_CUDA(ctx, cudaStreamSynchronize(ctx->last_stream));
+  const int S = (int)ctx->smids.size();
+  std::vector<unsigned long long> t((size_t)S * ugk::kTimelineWords);
+  UG_CUDA(ctx, cudaMemcpy(t.data(), ctx->d_timeline, t.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost));
+  ugk::Ctrl c;
+  UG_CUDA(ctx, cudaMemcpy(&c, ctx->d_ctrl, sizeof(c), cudaMemcpyDeviceToHost));
+  auto rel = [&](unsigned long long v) { return v > c.t_start ? (float)((v - c.t_start) * 1e-6) : 0.f; };
+  for (int i = 0; i < S; ++i) {
+    const unsigned long long *w = &t[(size_t)i * ugk::kTimelineWords];
+    out[i * 5 + 0] = (float)w[0];
+    for (int k = 1; k < 5; ++k) out[i * 5 + k] = rel(w[k]);
+  }
+  *num_ctas = S;
+  return UGACHE_OK;
+}
+
 ugache_status ugache_last_launch_count(const ugache_ctx *ctx, int32_t *launches) {
   if (!ctx || !launches) return UGACHE_EINVAL;
   *launches = ctx->last_launches;
@@ -1656,6 +1702,7 @@ ugache_status ugache_destroy(ugache_ctx *ctx) {
     cudaFree(ctx->d_loc);
     cudaFree(ctx->d_slot_keys);
     cudaFree(ctx->d_ctrl);
+    cudaFree(ctx->d_timeline);
     cudaFree(ctx->d_buckets);
     cudaFree(ctx->d_keys_stage);
     cudaFree(ctx->d_out_stage);

@@ -325,6 +325,16 @@ class UGache:
         check(lib().ugache_last_batch_phases(self.ctx, ms), "ugache_last_batch_phases", self.ctx)
         return tuple(float(x) for x in ms)
 
+    def last_batch_timeline(self):
+        """Per-CTA role timeline of the last fused launch (ugache_last_batch_timeline): an
+        (SM count, 5) float array of [role source, CTA start, gather start, role done, CTA
+        done], ms from the kernel's start.  Needs enable_timing(True)."""
+        buf = (ctypes.c_float * (5 * 256))()
+        n = ctypes.c_int32()
+        check(lib().ugache_last_batch_timeline(self.ctx, buf, ctypes.byref(n)), "ugache_last_batch_timeline",
+              self.ctx)
+        return np.frombuffer(buf, dtype=np.float32, count=5 * n.value).reshape(n.value, 5).copy()
+
     def last_extract_path(self) -> str:
         """'split', 'fused', 'single_pass', 'random' or 'none' (ugache_last_extract_path)."""
         p = ctypes.c_int32()

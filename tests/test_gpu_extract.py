@@ -659,20 +659,29 @@ def test_single_pass_static_schedule_and_chunk_sizes(torch_cuda, monkeypatch, G,
 
 def test_stream_auto_with_peers(torch_cuda):
     """auto keeps the two-phase kernel when peer rows are queued to dedicated SMs (G > 1,
-    default) and takes the single pass once peers are inline; both bit-exact."""
+    default, batches above 32768 keys) and takes the single pass once peers are inline or the
+    batch is small; all bit-exact."""
     N, R = 200_000, 512
     h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(51).permutation(N)]
     # partition of 2 x 95,000 rows: 5 % of uniform keys go to the host (a sparse bucket)
     t, group = make_group(torch_cuda, N, R, 95_000, 2, h, policy="partition")
     c = group[0]
     c.set_stream("auto")
-    keys = np.random.default_rng(52).integers(0, N, 30_000)
+    keys = np.random.default_rng(52).integers(0, N, 40_000)
     for peers_inline, want in ((False, "fused"), (True, "single_pass")):
         c.set_inline(host=True, peers=peers_inline)
         for _ in range(2):
             per = check_batch(torch_cuda, c, t, keys, N, R, 2)
             assert per[1] > 0 and 0 < per[2] < 3000, per
         assert c.last_extract_path() == want
+    # a small batch (<= 32768 keys, latency-bound) takes the single pass with its peer rows
+    # read inline even when peers are otherwise queued to dedicated SMs
+    c.set_inline(host=True, peers=False)
+    for n in (1, 8_192, 32_768):
+        per = check_batch(torch_cuda, c, t, keys[:n], N, R, 2)
+        assert c.last_extract_path() == "single_pass", n
+    check_batch(torch_cuda, c, t, keys[:32_769], N, R, 2)
+    assert c.last_extract_path() == "fused"
     for g in group:
         g.close()
 

@@ -97,6 +97,9 @@ def main():
     ap.add_argument("--table", default="")
     ap.add_argument("--summarize", default="", help="only rebuild --table from this JSONL file")
     ap.add_argument("--phases", action="store_true", help="record the fused kernel's phase stamps")
+    ap.add_argument("--batch-n", type=int, default=0, help="override the workload's keys (or samples) per batch")
+    ap.add_argument("--random", action="store_true",
+                    help="also time random dispatch (unfactored) on the same contexts and batches")
     args = ap.parse_args()
     if args.summarize:
         rows = [json.loads(x) for x in open(args.summarize) if x.strip()]
@@ -120,6 +123,8 @@ def main():
     nb = args.steps + 2
     for alpha in args.alphas:
         wl = dataclasses.replace(wl0, alpha=alpha)
+        if args.batch_n:
+            wl = dataclasses.replace(wl, batch_n=args.batch_n)
         t0 = time.time()
         h = synth.hotness(wl)
         keys_np = [synth.make_batch(wl, 0, b) for b in range(nb)]
@@ -171,6 +176,20 @@ def main():
                                     except Exception:  # noqa: BLE001 - single pass has no stamps
                                         phases.append(None)
                         path = cc.last_extract_path()
+                        rnd = []
+                        if args.random:
+                            cc.set_mode("random")
+                            for i in range(nb):
+                                flush.fill_(i & 0xFF)
+                                torch.cuda._sleep(100_000)
+                                s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                                s.record()
+                                cc.extract(keys[i], out)
+                                e.record()
+                                torch.cuda.synchronize()
+                                if i >= 2:
+                                    rnd.append(s.elapsed_time(e))
+                            cc.set_mode("factored")
                         cc.extract(keys[0], out)
                         torch.cuda.synchronize()
                         exact = bool(np.array_equal(out.cpu().numpy(), ref0))
@@ -185,6 +204,8 @@ def main():
                                  setup_s=time.time() - t1)
                         if args.phases:
                             r["phases_ms"] = phases
+                        if rnd:
+                            r["random_dispatch_ms"] = statistics.mean(rnd)
                         done[sig] = r
                         for g in group:
                             g.close()
