@@ -382,6 +382,28 @@ def config_dict(args, wl, ws):
             "batches": getattr(args, "batches", None)}
 
 
+def role_summary(tl, num_gpus, rank):
+    """Per-role view of the last fused launch's per-CTA timeline (ugache_last_batch_timeline):
+    CTAs per role and median / max of gather start, role done and CTA done, in us from the
+    kernel's start -- which source's SMs bound the batch (the paper's Fig. 8 picture)."""
+    roles = {}
+    for row in tl:
+        src = int(row[0])
+        name = "host" if src == num_gpus else ("local" if src == rank else f"peer{src}")
+        roles.setdefault(name, []).append(row)
+    out = {}
+    for name, rows in sorted(roles.items()):
+        a = np.array(rows) * 1e3
+        out[name] = {"ctas": len(rows),
+                     "gather_start": [round(float(np.median(a[:, 2])), 2), round(float(a[:, 2].max()), 2)],
+                     "role_done": [round(float(np.median(a[:, 3])), 2), round(float(a[:, 3].max()), 2)],
+                     "cta_done": [round(float(np.median(a[:, 4])), 2), round(float(a[:, 4].max()), 2)]}
+    out["how"] = ("per-CTA %globaltimer stamps of the last timed fused launch (rank 0): [median, max] "
+                  "us from the kernel's start; role_done = the CTA's own source drained, cta_done "
+                  "= after local padding")
+    return out
+
+
 def main():
     args = parse()
     launch_ranks(args)
@@ -600,7 +622,7 @@ def main():
 
     # kernel pass (steady state too: no flush): the library's own events around its launch
     # and the fused kernel's %globaltimer phase split, for the per-kernel roofline
-    loc_ms, gat_ms, phases = [], [], []
+    loc_ms, gat_ms, phases, timeline = [], [], [], None
     cache.enable_timing(True)
     for i in range(args.steps):
         cache.extract(dkeys[next_batch()], out, stream)
@@ -609,8 +631,10 @@ def main():
         gat_ms.append(b)
         if cache.last_extract_path() == "fused":
             phases.append(cache.last_batch_phases())
+            timeline = cache.last_batch_timeline()
     stream.synchronize()
     cache.enable_timing(False)
+    role_timeline = role_summary(timeline, ws, rank) if phases else None
     log("per-step ms (steady state): " + " ".join(f"{x:.3f}" for x in step_ms))
 
     # ---- cold L2: the same steps with a 256 MiB flush + ~50 us spin before each -----------
@@ -863,7 +887,7 @@ def main():
                                        "/ BW_HBM, NVLink ingress / BW_NVL, NVLink egress (rows peers read "
                                        "from g) / BW_NVL, host rows / BW_PCIe(g)); t_step = mean over steps "
                                        "of the max over ranks"},
-        "per_source_keys": {"local": n_local, "peer": n_peer, "host": n_host},
+        "per_source_keys": {"local": round(n_local, 2), "peer": round(max(n_peer, 0.0), 2), "host": round(n_host, 2)},
         "per_rank": ({"keys_from_source": P.tolist(), "kernel_ms": kern_all.tolist(),
                       "step_ms": step_all.tolist(), "pcie_peak_gbs": pcie_all.tolist(),
                       "t_roof_us": [r_["t_roof_s"] * 1e6 for r_ in rl["ranks"]]} if ws > 1 else None),
@@ -886,6 +910,7 @@ def main():
                              "launch_end": statistics.mean(p[4] for p in phases),
                              "how": "%globaltimer stamps inside the fused kernel, ms from its start"}
                             if phases else None),
+        "role_timeline_us": role_timeline,
         "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": n * 8,
                 "d2h_bytes_per_step": stats_bytes, "ms_per_step": statistics.mean(e2e_ms),
                 "path": "UGache.extract(pinned host keys -> HBM rows) + ugache_last_batch_stats "

@@ -80,3 +80,22 @@ def test_world_size_mismatch_is_an_error():
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "4", "--print-world"],
                        cwd=ROOT, env=env, capture_output=True, text=True, timeout=300)
     assert r.returncode == 2 and "WORLD_SIZE" in r.stderr
+
+
+def test_role_summary_groups_ctas_by_source():
+    """bench.role_summary: rows [role, start, gather, role done, done] (ms) are grouped by
+    source (this rank = local, num_gpus = host, other ids = peers), counted, and reported as
+    [median, max] in us."""
+    sys.path.insert(0, ROOT)
+    import numpy as np
+    import bench
+    tl = np.array([[2, 0.0, 0.010, 0.100, 0.120],    # host (G = 2)
+                   [2, 0.0, 0.012, 0.300, 0.310],
+                   [1, 0.0, 0.011, 0.020, 0.200],    # peer 1
+                   [0, 0.0, 0.010, 0.011, 0.150]],   # local (rank 0)
+                  dtype=np.float32)
+    r = bench.role_summary(tl, 2, 0)
+    assert r["host"]["ctas"] == 2 and r["peer1"]["ctas"] == 1 and r["local"]["ctas"] == 1
+    assert r["host"]["role_done"] == [200.0, 300.0]
+    assert r["local"]["cta_done"] == [150.0, 150.0]
+    assert r["peer1"]["gather_start"] == [11.0, 11.0]

@@ -755,6 +755,44 @@ def test_sparse_host_bucket_walk_or_order(torch_cuda, G):
         g.close()
 
 
+@pytest.mark.parametrize("G", [1, 4])
+def test_role_timeline(torch_cuda, G):
+    """ugache_last_batch_timeline after a fused launch: one row per SM; role counts match
+    the dedication (host CTAs = calibrated host SMs for a dense bucket, peer_sms per peer,
+    the rest local); per CTA start <= gather start <= role done <= done <= the launch end;
+    ESTATE after a single-pass launch or with timing off."""
+    from paper_conf_sosp_songz0c23_b200._abi import UGacheError
+    N, R = 300_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(66).permutation(N)]
+    t, group = make_group(torch_cuda, N, R, 20_000, G, h)
+    c = group[0]
+    c.set_stream("off")
+    keys = np.random.default_rng(67).integers(0, N, 200_000)     # dense host bucket
+    c.enable_timing(False)
+    check_batch(torch_cuda, c, t, keys, N, R, G)
+    with pytest.raises(UGacheError):
+        c.last_batch_timeline()
+    c.enable_timing(True)
+    check_batch(torch_cuda, c, t, keys, N, R, G)
+    tl = c.last_batch_timeline()
+    end = c.last_batch_phases()[4]
+    S = torch_cuda.cuda.get_device_properties(0).multi_processor_count
+    assert tl.shape == (S, 5)
+    roles = tl[:, 0].astype(int)
+    assert set(roles.tolist()) <= set(range(G + 1))
+    assert (roles == G).sum() == c.plan.host_sms
+    for j in range(1, G):
+        assert (roles == j).sum() == c.plan.peer_sms, (j, (roles == j).sum())
+    assert np.all(tl[:, 1] <= tl[:, 2]) and np.all(tl[:, 2] <= tl[:, 3]) and np.all(tl[:, 3] <= tl[:, 4])
+    assert tl[:, 4].max() <= end + 1e-3
+    c.set_stream("on")
+    check_batch(torch_cuda, c, t, keys[:5000], N, R, G)
+    with pytest.raises(UGacheError):
+        c.last_batch_timeline()
+    for g in group:
+        g.close()
+
+
 def test_fused_phase_stamps(torch_cuda):
     """ugache_last_batch_phases: after a fused launch with a dense host bucket the stamps are
     ordered (locate <= host ordered <= host copies done <= the launch's event time); after a
