@@ -595,10 +595,25 @@ __device__ __forceinline__ void preorder_host(const GatherParams &p, uint32_t *s
   block_exclusive_scan(p.range_count, s_tab, p.n_ranges);
   const uint64_t *b = p.buckets + (uint64_t)host_src * p.bucket_cap;
   const uint32_t lo = (uint32_t)((uint64_t)cnt * pos / S), hi = (uint32_t)((uint64_t)cnt * (pos + 1) / S);
+  // The CTA reserves one block per non-empty range (one global atomic per (CTA, range)
+  // instead of one per entry: the hot head of the tier puts thousands of a batch's host
+  // keys in its first ranges, and per-entry atomics on their cursors serialised), then
+  // places its entries with shared-memory cursors.  s_loc lives in the first TMA staging
+  // buffers, idle until the gather starts (after this function's last barrier).
+  uint32_t *s_loc = s_tab + kMaxRanges;
+  for (uint32_t i = tid; i < p.n_ranges; i += blockDim.x) s_loc[i] = 0;
+  __syncthreads();
+  for (uint32_t e = lo + tid; e < hi; e += blockDim.x)
+    atomicAdd(&s_loc[(uint32_t)(b[e] >> 32) >> p.range_shift], 1u);
+  __syncthreads();
+  for (uint32_t i = tid; i < p.n_ranges; i += blockDim.x) {
+    const uint32_t c = s_loc[i];
+    if (c) s_loc[i] = s_tab[i] + atomicAdd(&p.range_cursor[i], c);
+  }
+  __syncthreads();
   for (uint32_t e = lo + tid; e < hi; e += blockDim.x) {
     const uint64_t ent = b[e];
-    const uint32_t r = (uint32_t)(ent >> 32) >> p.range_shift;
-    p.host_sorted[s_tab[r] + atomicAdd(&p.range_cursor[r], 1u)] = ent;
+    p.host_sorted[atomicAdd(&s_loc[(uint32_t)(ent >> 32) >> p.range_shift], 1u)] = ent;
   }
   __syncthreads();
   if (tid == 0) {
