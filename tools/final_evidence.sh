@@ -4,7 +4,7 @@
 # fused kernel on gnn_pa@0.25 (kernel replay; the full-size tier cannot be saved/restored).
 o=${1:-gpurun_out/final}; mkdir -p $o
 bash tools/gpu_round_check.sh $o
-timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"extract|random_dispatch|fill" -c 120 --csv \
+timeout 900 ncu --replay-mode application --metrics gpu__time_duration.sum --clock-control none -k regex:"extract|random_dispatch|fill" -c 120 --csv \
   --log-file $o/launches_default.csv python bench.py --steps 3 --warmup 3 > $o/ncu_launches.log 2>&1; echo "launches rc $?"
 timeout 1500 ncu --replay-mode application --clock-control none \
   --metrics dram__bytes_read.sum,dram__bytes_write.sum,pcie__read_bytes.sum,pcie__read_bytes.sum.per_second,gpu__time_duration.sum \
