@@ -439,7 +439,8 @@ ugache_status ugache_last_batch_phases(ugache_ctx *ctx, float *ms);
 /* Per-CTA role timeline of the last fused (K1+K2) launch, for the paper's per-source time
  * split (Fig. 8's picture; §5.3): one CTA per SM, listed in the chip-spreading
  * order the roles are assigned in.  out[5*i .. 5*i+4] for position i = {role source id (GPU
- * j = peer j or this rank = local, num_gpus = host), CTA start, gather start (grid barrier
+ * j = peer j or this rank = local, num_gpus = host, num_gpus + 1 = warp-granular dedication:
+ * every SM mixes roles; the role-done stamp is then 0), CTA start, gather start (grid barrier
  * and host pre-ordering done), own role done (local padding follows), CTA done}, times in
  * ms from the kernel's start.  out: caller-owned, 5 * (SM count) floats (<= 5 * 256);
  * *num_ctas = SM count.  Needs ugache_enable_timing(ctx, 1) before the extract (the stamps

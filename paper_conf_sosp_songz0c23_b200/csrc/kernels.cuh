@@ -869,6 +869,7 @@ __device__ __forceinline__ void gather_body(const GatherParams &p, uint32_t *s_d
   bool host_cta = false;  // SM-granular mode: this CTA holds a host role
 
   if (p.warp_dedication) {
+    if (tl && threadIdx.x == 0) tl[0] = (unsigned long long)p.num_src;  // mixed roles (timeline)
     // Warp-granular dedication: on EVERY SM, warps [0, hw) serve the
     // host and the next pw warps each peer; the rest start on local work.  Concurrency per
     // slow source stays bounded (S*hw or S*pw warps) while the requests come from all GPCs
