@@ -389,7 +389,8 @@ def role_summary(tl, num_gpus, rank):
     roles = {}
     for row in tl:
         src = int(row[0])
-        name = "host" if src == num_gpus else ("local" if src == rank else f"peer{src}")
+        name = ("host" if src == num_gpus else "mixed" if src == num_gpus + 1
+                else "local" if src == rank else f"peer{src}")
         roles.setdefault(name, []).append(row)
     out = {}
     for name, rows in sorted(roles.items()):

@@ -22,7 +22,7 @@ def summarize(tl, G, rank=0):
     roles = {}
     for row in tl:
         src = int(row[0])
-        name = "host" if src == G else ("local" if src == rank else f"peer{src}")
+        name = "host" if src == G else "mixed" if src == G + 1 else ("local" if src == rank else f"peer{src}")
         roles.setdefault(name, []).append(row)
     out = {}
     for name, rows in sorted(roles.items()):
