@@ -86,6 +86,7 @@ def parse():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--workload", default="gnn_pa")
     ap.add_argument("--cache-ratio", type=float, default=None)
+    ap.add_argument("--alpha", type=float, default=None, help="Zipf alpha (default: the workload's)")
     ap.add_argument("--policy", default="ugache")
     ap.add_argument("--mode", default="factored", choices=["factored", "random"])
     ap.add_argument("--stream", default="auto", choices=["off", "on", "auto"],
@@ -418,6 +419,9 @@ def main():
     if args.cache_ratio is not None:
         from dataclasses import replace
         wl = replace(wl, cache_ratio=args.cache_ratio)
+    if args.alpha is not None:   # Zipf skew of the keys and hotness (GNN 1.2 plus 1.4)
+        from dataclasses import replace
+        wl = replace(wl, alpha=args.alpha)
     if args.impl == "reference":
         run_reference(args, wl)
         return

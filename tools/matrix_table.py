@@ -23,7 +23,8 @@ for f in sorted(os.listdir(d)):
     cold = j.get("cold_l2") or {}
     rr = r.get("random_row_peak") or {}
     rows.append("| {} | {} | {:.0%} | {} | {:.4f} | {:.0f} | {} {:.2f} | {} | {:.4f} | {} | {} | {} | {} | {} |".format(
-        c["workload"], c["keys_per_batch_per_gpu"], c["cache_ratio"], r.get("path"), j["ms_per_step"], j["value"],
+        c["workload"] + (f" (alpha {c['alpha']:g})" if c.get("alpha", 1.2) != 1.2 else ""),
+        c["keys_per_batch_per_gpu"], c["cache_ratio"], r.get("path"), j["ms_per_step"], j["value"],
         r["term"], r["frac"], f"{rr['frac']:.2f}" if rr else "-",
         cold.get("ms_per_step", float("nan")), f"{cold['roofline_frac']:.2f}" if cold.get("roofline_frac") else "-",
         f"{ps['host'] / n:.1%}",
