@@ -1642,6 +1642,62 @@ __global__ void __launch_bounds__(kGatherThreads, 1)
   stream_body<KeyT>(lp, gp, s_dyn, pos);
 }
 
+// ---------------------------------------------------------------------------- K3r
+// Single pass, register variant, for batches whose every source is read inline (no queued
+// source: G = 1 or peers inline) and whose host bucket is sparse (cold host rows, latency-
+// bound).  Each warp takes chunks of stream_ck (<= 32) keys on the
+// static schedule, locates them, and copies its rows RegRows at a time straight from the
+// lanes that located them (no copy list in shared memory, no TMA slots, no queue
+// bookkeeping): a lean kernel whose registers leave room for 8 rows in flight per warp
+// step and two CTAs per SM.  Same output, same per-source counts as K3.
+constexpr int kRegRows = 8;
+template <typename KeyT>
+__global__ void __launch_bounds__(kGatherThreads, 2)
+    stream_extract_reg_kernel(const LocateParams lp, const GatherParams gp) {
+  __shared__ uint32_t s_inl[kMaxSrc];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x < kMaxSrc) s_inl[threadIdx.x] = 0;
+  __syncthreads();
+  const uint32_t n = lp.n, ck = (uint32_t)gp.stream_ck, R = gp.row_bytes;
+  const uint32_t nchunks = (n + ck - 1) / ck;
+  const uint32_t W = gridDim.x * (blockDim.x >> 5);
+  const KeyT *keys = static_cast<const KeyT *>(lp.keys);
+  uint32_t nbad = 0;
+  for (uint32_t c = blockIdx.x * (blockDim.x >> 5) + warp; c < nchunks; c += W) {
+    const uint32_t i = c * ck + (uint32_t)lane;
+    int s = -1;
+    uint64_t a = 0;
+    if ((uint32_t)lane < ck && i < n) {
+      const KeyT k = keys[i];
+      if (key_in_range<KeyT>(k, lp.num_rows)) {
+        const uint64_t e = ld_lt_u64(lp.loc + (uint64_t)k);
+        s = (int)(e >> UGACHE_LOC_SRC_SHIFT);
+        a = reinterpret_cast<uint64_t>(gp.base[s]) + (e & UGACHE_LOC_ROW_MASK) * (uint64_t)R;
+      } else {
+        zero_row(gp.out + (uint64_t)i * R, R);  // out-of-range key
+        ++nbad;
+      }
+    }
+    const uint32_t peers = __match_any_sync(kFullMask, s);
+    if (s >= 0 && lane == __ffs(peers) - 1) atomicAdd(&s_inl[s], (uint32_t)__popc(peers));
+    // rows of this chunk, kRegRows per step, taken from the lanes that located them
+    const uint32_t m = __ballot_sync(kFullMask, s >= 0);
+    const int nrows = __popc(m);
+    for (int g0 = 0; g0 < nrows; g0 += kRegRows) {
+      const int nv = min(kRegRows, nrows - g0);
+      // lane u < nv takes the (g0 + u)-th located lane's row
+      const int srcl = lane < nv ? (int)__fns(m, 0, g0 + lane + 1) : 0;
+      const uint64_t au = __shfl_sync(kFullMask, a, srcl);
+      const uint32_t ou = c * ck + (uint32_t)srcl;
+      copy_addr_rows<kRegRows>(gp.out, R, au, ou, nv, lane);
+    }
+  }
+  if (nbad) atomicAdd(&gp.ctrl->bad, nbad);
+  __syncthreads();
+  if (threadIdx.x < gp.num_src && s_inl[threadIdx.x]) atomicAdd(&gp.ctrl->counts[threadIdx.x], s_inl[threadIdx.x]);
+  finish_launch(gp.ctrl, gp.num_src, n, 1);
+}
+
 // ---------------------------------------------------------------------------- K2'
 template <typename KeyT>
 __global__ void __launch_bounds__(kGatherThreads, 1)

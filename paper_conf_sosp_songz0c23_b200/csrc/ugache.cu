@@ -84,6 +84,8 @@ struct ugache_ctx {
   int host_segments = 2;                     // env UGACHE_HOST_SEGMENTS (ordered host copy)
   int locate_spread = 1;                     // env UGACHE_LOCATE_SPREAD (fused: tile size from n)
   int local_pace = 0;                        // env UGACHE_LOCAL_PACE (ns, experiment)
+  int reg_kernel_ck = 8;                     // env UGACHE_REG_KERNEL_CK: keys per chunk of K3r (sparse
+                                             // host, every source inline); 0 = K3's register path
   uint64_t small_batch_keys = 32768;         // env UGACHE_SMALL_BATCH: auto path reads peers inline
                                              // in the single pass up to this many keys
   uint64_t walk_keys_per_sm = 1024;          // env UGACHE_WALK_KEYS_PER_SM: a sparse host bucket is
@@ -485,6 +487,10 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
     UG_CUDA(ctx, cudaMemcpyToSymbol(ugk::c_lt_evict_first, &lf, sizeof(lf)));
   }
   if (const char *e = getenv("UGACHE_INLINE")) ctx->inline_mask = atoi(e) & (UGACHE_INLINE_HOST | UGACHE_INLINE_PEERS);
+  if (const char *e = getenv("UGACHE_REG_KERNEL_CK")) {
+    const int v = atoi(e);
+    ctx->reg_kernel_ck = v <= 0 ? 0 : v <= 8 ? 8 : v <= 16 ? 16 : 32;
+  }
   if (const char *e = getenv("UGACHE_SMALL_BATCH")) ctx->small_batch_keys = strtoull(e, nullptr, 10);
   if (const char *e = getenv("UGACHE_WALK_KEYS_PER_SM")) ctx->walk_keys_per_sm = strtoull(e, nullptr, 10);
   if (const char *e = getenv("UGACHE_STREAM_GROUP"))
@@ -1374,6 +1380,7 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
       }
     }
     const bool fused = ctx->fused == 1 || (ctx->fused == 2 && n <= kFusedAutoMaxKeys);
+    bool reg_kernel = false;
     if (stream && ctx->sparse_host_regpath && exp_host >= 0.005 * (double)n && ctx->stream_ck == 0) {
       // a sparse but present host bucket (cold host rows, latency-bound): the register path
       // with 16-key chunks keeps fewer host requests in flight per warp and measured faster
@@ -1381,6 +1388,10 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
       gp.stream_bulk = 0;
       gp.stream_ck = std::min<int32_t>(gp.stream_ck, 16);
       gp.stream_k = 1;
+      if (!gp.stream_queues && ctx->reg_kernel_ck > 0) {  // every source inline: the lean K3r
+        reg_kernel = true;
+        gp.stream_ck = ctx->reg_kernel_ck;
+      }
     }
     if (!stream && ctx->preorder && ctx->host_sort && !gp.early_walk) {
       // two-phase paths: the locate pass builds the host range histogram, and every CTA of the
@@ -1396,7 +1407,11 @@ ugache_status extract_impl(ugache_ctx *ctx, const void *keys, int32_t key_type, 
       void *kargs[] = {&lp, &gp};
       const void *fn = key_type == UGACHE_KEY_I64 ? (const void *)ugk::stream_extract_kernel<int64_t>
                                                   : (const void *)ugk::stream_extract_kernel<uint32_t>;
-      if (gp.stream_queues || ctx->stream_coop) {
+      if (reg_kernel) {
+        const void *rf = key_type == UGACHE_KEY_I64 ? (const void *)ugk::stream_extract_reg_kernel<int64_t>
+                                                    : (const void *)ugk::stream_extract_reg_kernel<uint32_t>;
+        UG_CUDA(ctx, cudaLaunchKernel(rf, dim3(2 * ctx->sm_count), dim3(ugk::kGatherThreads), kargs, 0, s));
+      } else if (gp.stream_queues || ctx->stream_coop) {
         UG_CUDA(ctx, cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(ugk::kGatherThreads), kargs,
                                                  kOneCtaPerSmSmem, s));
       } else {  // no queues: no CTA waits on another, a plain launch is enough

@@ -793,6 +793,32 @@ def test_role_timeline(torch_cuda, G):
         g.close()
 
 
+@pytest.mark.parametrize("ck", ["8", "16", "32", "0"])
+@pytest.mark.parametrize("G", [1, 4])
+def test_single_pass_register_kernel(torch_cuda, monkeypatch, ck, G):
+    """K3r, the lean register single pass (sparse host bucket, every source inline;
+    UGACHE_REG_KERNEL_CK = keys per chunk, 0 = K3's own register path): bit-exact with
+    out-of-range keys, both key types, ragged and tiny batches, G = 1 and G = 4 with peer
+    rows inline; per-source counts exact."""
+    monkeypatch.setenv("UGACHE_REG_KERNEL_CK", ck)
+    N, R = 200_000, 512
+    h = (synth.zipf_pmf(N, 1.2) * 1e5).astype(np.float32)[np.random.default_rng(68).permutation(N)]
+    t, group = make_group(torch_cuda, N, R, 190_000 // G, G, h, policy="partition")
+    c = group[0]
+    c.set_stream("auto")
+    c.set_inline(host=True, peers=True)
+    rng = np.random.default_rng(69)
+    for n in (1, 33, 8_191, 50_000, 70_001):
+        keys = rng.integers(-3, N + 3, n)
+        for kd in (np.int64, np.uint32):
+            per = check_batch(torch_cuda, c, t, np.abs(keys) if kd == np.uint32 else keys, N, R, G, key_dtype=kd)
+            if n >= 50_000:
+                assert 0.005 * n <= per[G] < 4096, per
+                assert c.last_extract_path() == "single_pass"
+    for g in group:
+        g.close()
+
+
 def test_fused_phase_stamps(torch_cuda):
     """ugache_last_batch_phases: after a fused launch with a dense host bucket the stamps are
     ordered (locate <= host ordered <= host copies done <= the launch's event time); after a
