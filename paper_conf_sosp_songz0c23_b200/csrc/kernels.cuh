@@ -8,6 +8,8 @@
 //  K3 stream_extract_kernel : single pass -- chunks located and copied at once through
 //                            per-lane TMA slots; queued sources drained by their dedicated
 //                            SMs from per-CTA sub-queues (no grid barrier, no local bucket)
+//  K3r stream_extract_reg_kernel : single pass, register variant for a sparse host bucket
+//                            with every source inline (8-key chunks, 8 rows per warp step)
 //  K2' random_dispatch_kernel : unfactored peer-based baseline, ablation only
 //  K5 fill_kernel          : Filler, host rows -> this GPU's cache slab
 //
