@@ -1,3 +1,5 @@
+# NOTE: UGACHE_STREAM_REG_ROWS (K3 register path rows per step) was measured here and then removed
+# (no gain, register spills); K3r (stream_extract_reg_kernel) replaced it -- profiles/r2/k3r/.
 # Single pass with a sparse host bucket (G = 1): keys per chunk (UGACHE_STREAM_CK) x register
 # rows per step, against random dispatch (gnn_pa@0.25 at 20K / 100K keys, DLR@0.15).
 o=${1:-gpurun_out/ck}; mkdir -p $o

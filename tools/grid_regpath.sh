@@ -1,3 +1,5 @@
+# NOTE: UGACHE_STREAM_REG_ROWS (K3 register path rows per step) was measured here and then removed
+# (no gain, register spills); K3r (stream_extract_reg_kernel) replaced it -- profiles/r2/k3r/.
 # Single pass with a sparse host bucket (G = 1): register path 4 vs 8 rows per step, TMA
 # slots, and random dispatch, at 20K / 100K / 213K-key batches (gnn_pa@0.25, alpha 1.2).
 o=${1:-gpurun_out/regpath}; mkdir -p $o
