@@ -489,7 +489,7 @@ ugache_status init_common(ugache_ctx *ctx, const ugache_config *cfg, const void 
   if (const char *e = getenv("UGACHE_INLINE")) ctx->inline_mask = atoi(e) & (UGACHE_INLINE_HOST | UGACHE_INLINE_PEERS);
   if (const char *e = getenv("UGACHE_REG_KERNEL_CK")) {
     const int v = atoi(e);
-    ctx->reg_kernel_ck = v <= 0 ? 0 : v <= 8 ? 8 : v <= 16 ? 16 : 32;
+    ctx->reg_kernel_ck = v <= 0 ? 0 : v <= 4 ? 4 : v <= 8 ? 8 : v <= 16 ? 16 : 32;
   }
   if (const char *e = getenv("UGACHE_SMALL_BATCH")) ctx->small_batch_keys = strtoull(e, nullptr, 10);
   if (const char *e = getenv("UGACHE_WALK_KEYS_PER_SM")) ctx->walk_keys_per_sm = strtoull(e, nullptr, 10);
